@@ -1,0 +1,162 @@
+/*
+ * ds.h -- libds: in-place Data Sliding (DS) primitives on NVIDIA B200 (sm_100a).
+ *
+ * C ABI of the hot path.  Every call runs hand-written CUDA kernels; there is
+ * no CPU fallback.  "P:NN" cites line NN of the paper text PAPER.md
+ * (Gomez-Luna, Chang, Sung, Hwu, Guil, "In-Place Data Sliding Algorithms for
+ * Many-Core Architectures", ICPP 2015).  Readings "Rnn" are listed in
+ * DESIGN.md section 3.
+ *
+ * Common contract
+ *  - Pointers named `ptr` are DEVICE memory on the CURRENT CUDA device
+ *    (cudaMalloc'd or a torch tensor's data_ptr()), owned by the caller.
+ *    libds never frees, reallocates or keeps them, and never allocates
+ *    an n-sized scratch buffer (the operations are in place).
+ *  - `ptr` must be 4-byte aligned; 16-byte alignment is not required.
+ *  - Words are 32-bit; compact/select/unique compare bit patterns (R13),
+ *    so they serve int32, uint32 and float32 arrays alike.
+ *  - All argument validation happens BEFORE anything is launched: on any
+ *    DS_ERROR_INVALID_VALUE / DS_ERROR_UNSUPPORTED return the buffer and
+ *    the output count are untouched.  DS_ERROR_CUDA means a CUDA call
+ *    failed after launch; the buffer content is then undefined (in place).
+ *  - Kept outputs are stable.  Words in [out_n, n) (compact/select/
+ *    unique) and in [rows*new_cols, rows*cols) elements (unpad) are left
+ *    exactly as they were (R5).
+ *  - The plain forms run on the legacy default stream and BLOCK until the
+ *    result (and *out_n) is known.  The _ex forms are asynchronous and
+ *    stream-ordered on `stream`; their count is written to DEVICE memory
+ *    (d_out_n, may be NULL).
+ *  - libds keeps, per (device, stream), a small workspace: one 64-bit
+ *    status word per tile (n/4096 words, ~0.2% of the data) and one
+ *    ticket/epoch word.  Calls that share a stream share it; calls on
+ *    different streams may run concurrently.  ds_release_workspaces()
+ *    frees it (call only when no libds kernel is in flight).
+ *  - Thread-safe: host state is protected by a mutex.
+ */
+#ifndef LIBDS_DS_H
+#define LIBDS_DS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Same object as cudaStream_t / CUstream; NULL = legacy default stream. */
+typedef struct CUstream_st* ds_stream_t;
+
+typedef enum ds_status {
+    DS_SUCCESS = 0,
+    DS_ERROR_INVALID_VALUE = 1, /* NULL pointer, misaligned ptr, bad sizes  */
+    DS_ERROR_UNSUPPORTED = 2,   /* valid but not implemented (elem_bytes 1/2,
+                                   n >= 2^36 words, rows longer than 2^30 words) */
+    DS_ERROR_OUT_OF_MEMORY = 3, /* workspace allocation failed              */
+    DS_ERROR_CUDA = 4           /* a CUDA runtime call failed               */
+} ds_status;
+
+/* Select predicates (Fig. 11's example "element value is even",
+ * P:238).  ds_select KEEPS the words for which the predicate is TRUE (R14);
+ * "remove if p" is the complementary id.  `param` is a 32-bit pattern.   */
+typedef enum ds_predicate {
+    DS_PRED_NONZERO = 0,    /* w != 0 (bitwise)                                */
+    DS_PRED_I32_GT = 1,     /* (int32)w >  (int32)param                       */
+    DS_PRED_I32_NOT_GT = 2, /* !((int32)w > (int32)param)                     */
+    DS_PRED_F32_GT = 3,     /* (float)w >  (float)param; NaN -> false (R16)   */
+    DS_PRED_F32_NOT_GT = 4, /* !((float)w > (float)param); NaN -> true        */
+    DS_PRED_I32_EVEN = 5,   /* (int32)w is even                               */
+    DS_PRED_I32_ODD = 6,    /* (int32)w is odd                                */
+    DS_PRED_COUNT = 7
+} ds_predicate;
+
+/* ---------------------------------------------------------------------
+ * Regular DS (Algorithm 1)
+ * ------------------------------------------------------------------- */
+
+/* ds_pad -- padding matrix columns in place.
+ * ptr: row-major rows x cols matrix of elem_bytes-sized elements, in a
+ *      buffer the CALLER made at least rows*new_cols*elem_bytes long ("the
+ *      extra memory space needs to be previously allocated adjacent to the
+ *      matrix"; cannot be checked, R4).
+ * After the call ptr holds rows x new_cols: row i moved forward by
+ * (new_cols-cols)*i elements ("row i will be shifted by C x i") and
+ * followed by new_cols-cols fill elements (zero bytes, R1/R2).
+ * Requires new_cols >= cols; elem_bytes in {4, 8, 16}.                   */
+ds_status ds_pad(void* ptr, size_t rows, size_t cols, size_t new_cols,
+                 size_t elem_bytes);
+
+/* ds_unpad -- "removes the extra columns": keeps the first
+ * new_cols elements of every row; rows move backward.  new_cols <= cols.  */
+ds_status ds_unpad(void* ptr, size_t rows, size_t cols, size_t new_cols,
+                   size_t elem_bytes);
+
+/* Asynchronous forms.  fill: HOST pointer to elem_bytes bytes copied into
+ * every new cell (NULL = zero bytes).                                    */
+ds_status ds_pad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols,
+                    size_t elem_bytes, const void* fill, ds_stream_t stream);
+ds_status ds_unpad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols,
+                      size_t elem_bytes, ds_stream_t stream);
+
+/* ---------------------------------------------------------------------
+ * Irregular DS (Algorithm 2)
+ * ------------------------------------------------------------------- */
+
+/* ds_compact -- stream compaction: removes the words equal
+ * (bitwise) to remove_value, keeps the others in order at ptr[0, *out_n).
+ * out_n: HOST pointer, required.                                         */
+ds_status ds_compact(void* ptr, size_t n, uint32_t remove_value, size_t* out_n);
+
+/* ds_select -- select with predicate_id (ds_predicate) and
+ * param = 0; keeps predicate-true words at ptr[0, *out_n).               */
+ds_status ds_select(void* ptr, size_t n, int predicate_id, size_t* out_n);
+
+/* ds_unique -- unique: word i is kept iff i == 0 or
+ * w[i] != w[i-1] (bitwise, original values, R13).                 */
+ds_status ds_unique(void* ptr, size_t n, size_t* out_n);
+
+/* Asynchronous forms; d_out_n: DEVICE pointer receiving the kept count
+ * (uint64), or NULL.                                                     */
+ds_status ds_compact_ex(void* ptr, size_t n, uint32_t remove_value,
+                        uint64_t* d_out_n, ds_stream_t stream);
+ds_status ds_select_ex(void* ptr, size_t n, int predicate_id, uint32_t param,
+                       uint64_t* d_out_n, ds_stream_t stream);
+/* d_halo / halo_len: for a shard of a longer array (R18).  DEVICE array of
+ * halo_len entries made by ds_halo_entry() for the shards BEFORE this one,
+ * in order; word 0 is compared with the last word of the nearest non-empty
+ * earlier shard (kept if there is none).  NULL/0 for a whole array.      */
+ds_status ds_unique_ex(void* ptr, size_t n, const uint64_t* d_halo,
+                       size_t halo_len, uint64_t* d_out_n, ds_stream_t stream);
+
+/* ---------------------------------------------------------------------
+ * Sharding helpers (multi-GPU).  Each GPU slides its
+ * own contiguous shard; NCCL all-gathers 8-byte values between the calls.
+ * ------------------------------------------------------------------- */
+
+/* d_entry[0] = (n > 0) << 32 | ptr[n-1]  -- the shard's halo entry for
+ * unique.  May be called before or after ds_unique_ex on the same shard:
+ * unique never changes ptr[n-1] (it is either untouched tail or kept).   */
+ds_status ds_halo_entry(const void* ptr, size_t n, uint64_t* d_entry,
+                        ds_stream_t stream);
+
+/* d_result[0] = sum(d_counts[0 .. rank)), d_result[1] = sum(d_counts[0 ..
+ * world)): this shard's global output offset and the global out_n.       */
+ds_status ds_shard_offsets(const uint64_t* d_counts, size_t world, size_t rank,
+                           uint64_t* d_result, ds_stream_t stream);
+
+/* ---------------------------------------------------------------------
+ * Utilities
+ * ------------------------------------------------------------------- */
+const char* ds_status_string(ds_status status);
+/* Message of the last failing CUDA call in this thread ("" if none).     */
+const char* ds_last_error(void);
+/* Frees every workspace of the calling process (all devices/streams).    */
+ds_status ds_release_workspaces(void);
+/* Number of kernel launches libds issued in this process (for bench.py). */
+uint64_t ds_launch_count(void);
+/* Library version, major*10000 + minor*100 + patch.                      */
+int ds_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LIBDS_DS_H */

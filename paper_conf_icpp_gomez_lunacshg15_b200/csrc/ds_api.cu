@@ -1,0 +1,317 @@
+// ds_api.cu -- the libds C ABI (include/ds.h): argument validation, the
+// per-(device, stream) workspace cache, dispatch to the kernels, and the
+// blocking wrappers.  Every validation happens before anything touches the
+// device, so an error return leaves the caller's buffer untouched.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <string>
+#include <utility>
+
+#include "ds.h"
+#include "ds_device.cuh"
+#include "ds_internal.h"
+
+namespace {
+
+constexpr uint64_t kMaxWords = (1ull << 36) - 1;     // status count field (36 bits)
+constexpr uint64_t kMaxRowWords = (1ull << 30);      // 32-bit in-tile column math
+constexpr uint64_t kMaxMatrixWords = (1ull << 42);   // tile ids stay 32-bit
+constexpr uint64_t kResetEvery = 1ull << 25;         // zero statuses before the 26-bit epoch wraps
+
+std::mutex g_mu;
+std::map<std::pair<int, uintptr_t>, ds::Workspace> g_ws;
+std::atomic<uint64_t> g_launches{0};
+thread_local std::string g_err;
+
+ds_status fail(cudaError_t e, const char* what) {
+    g_err = std::string(what) + ": " + cudaGetErrorString(e);
+    return DS_ERROR_CUDA;
+}
+
+bool misaligned(const void* p, uintptr_t a) { return (reinterpret_cast<uintptr_t>(p) & (a - 1)) != 0; }
+
+// Caller holds g_mu.
+ds_status get_workspace(size_t tiles, cudaStream_t s, ds::Workspace** out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return fail(e, "cudaGetDevice");
+    ds::Workspace& ws = g_ws[{dev, reinterpret_cast<uintptr_t>(s)}];
+    if (!ws.ctrl) {
+        // ctrl = {epoch 1, ticket 0}; d_count lives right after it.
+        if ((e = cudaMalloc(&ws.ctrl, 2 * sizeof(uint64_t))) != cudaSuccess) {
+            ws.ctrl = nullptr;
+            return e == cudaErrorMemoryAllocation ? DS_ERROR_OUT_OF_MEMORY : fail(e, "cudaMalloc");
+        }
+        const uint64_t init[2] = {1ull << 32, 0};
+        if ((e = cudaMemcpy(ws.ctrl, init, sizeof(init), cudaMemcpyHostToDevice)) != cudaSuccess)
+            return fail(e, "cudaMemcpy");
+        ws.d_count = ws.ctrl + 1;
+        if ((e = cudaMallocHost(&ws.h_count, sizeof(uint64_t))) != cudaSuccess)
+            return fail(e, "cudaMallocHost");
+    }
+    if (ws.cap_tiles < tiles) {
+        if (ws.status) {
+            // The old array may still be read by queued kernels of this stream.
+            if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return fail(e, "cudaStreamSynchronize");
+            cudaFree(ws.status);
+            ws.status = nullptr;
+            ws.cap_tiles = 0;
+        }
+        size_t cap = tiles < 1024 ? 1024 : tiles;
+        if ((e = cudaMalloc(&ws.status, cap * sizeof(uint64_t))) != cudaSuccess) {
+            ws.status = nullptr;
+            return e == cudaErrorMemoryAllocation ? DS_ERROR_OUT_OF_MEMORY : fail(e, "cudaMalloc");
+        }
+        ws.cap_tiles = cap;
+        ws.launches = kResetEvery;  // force the zeroing below
+    }
+    if (ws.launches >= kResetEvery) {
+        if ((e = cudaMemsetAsync(ws.status, 0, ws.cap_tiles * sizeof(uint64_t), s)) != cudaSuccess)
+            return fail(e, "cudaMemsetAsync");
+        ws.launches = 0;
+    }
+    ws.launches++;
+    *out = &ws;
+    return DS_SUCCESS;
+}
+
+ds_status run_irregular(const ds::IrregArgs& a, cudaStream_t s) {
+    std::lock_guard<std::mutex> lock(g_mu);
+    ds::Workspace* ws = nullptr;
+    ds_status st = get_workspace(ds::irregular_tiles(a), s, &ws);
+    if (st != DS_SUCCESS) return st;
+    cudaError_t e = ds::launch_irregular(a, *ws, s);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "irregular kernel launch");
+}
+
+ds_status check_irregular(const void* ptr, size_t n, const uint64_t* d_out_n) {
+    if (n > 0 && ptr == nullptr) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(ptr, 4) || misaligned(d_out_n, 8)) return DS_ERROR_INVALID_VALUE;
+    if (n > kMaxWords) return DS_ERROR_UNSUPPORTED;
+    return DS_SUCCESS;
+}
+
+ds_status irregular_ex(ds::IrregArgs a, cudaStream_t s) {
+    if (a.n == 0) {
+        if (a.d_out_n) {
+            cudaError_t e = cudaMemsetAsync(a.d_out_n, 0, sizeof(uint64_t), s);
+            if (e != cudaSuccess) return fail(e, "cudaMemsetAsync");
+        }
+        return DS_SUCCESS;
+    }
+    return run_irregular(a, s);
+}
+
+// Blocking form: legacy default stream, count read back through the
+// workspace's pinned mirror.
+ds_status irregular_blocking(ds::IrregArgs a, size_t* out_n) {
+    if (a.n == 0) {
+        *out_n = 0;
+        return DS_SUCCESS;
+    }
+    std::lock_guard<std::mutex> lock(g_mu);
+    cudaStream_t s = nullptr;
+    ds::Workspace* ws = nullptr;
+    ds_status st = get_workspace(ds::irregular_tiles(a), s, &ws);
+    if (st != DS_SUCCESS) return st;
+    a.d_out_n = ws->d_count;
+    cudaError_t e = ds::launch_irregular(a, *ws, s);
+    if (e != cudaSuccess) return fail(e, "irregular kernel launch");
+    if ((e = cudaMemcpyAsync(ws->h_count, ws->d_count, sizeof(uint64_t), cudaMemcpyDeviceToHost, s)) !=
+        cudaSuccess)
+        return fail(e, "cudaMemcpyAsync");
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return fail(e, "cudaStreamSynchronize");
+    *out_n = size_t(*ws->h_count);
+    return DS_SUCCESS;
+}
+
+ds_status check_regular(const void* ptr, size_t rows, size_t cols, size_t new_cols, size_t eb,
+                        bool pad, ds::RegArgs* a) {
+    if (eb == 1 || eb == 2) return DS_ERROR_UNSUPPORTED;
+    if (eb != 4 && eb != 8 && eb != 16) return DS_ERROR_INVALID_VALUE;
+    if (pad ? new_cols < cols : new_cols > cols) return DS_ERROR_INVALID_VALUE;
+    size_t big = pad ? new_cols : cols, tmp = 0;
+    if (__builtin_mul_overflow(rows, big, &tmp) || __builtin_mul_overflow(tmp, eb, &tmp))
+        return DS_ERROR_INVALID_VALUE;
+    if (tmp > 0 && ptr == nullptr) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(ptr, 4)) return DS_ERROR_INVALID_VALUE;
+    const uint64_t w = eb / 4;
+    if (uint64_t(big) * w >= kMaxRowWords) return DS_ERROR_UNSUPPORTED;
+    if (tmp / 4 > kMaxMatrixWords) return DS_ERROR_UNSUPPORTED;
+    a->ptr = static_cast<uint32_t*>(const_cast<void*>(ptr));
+    a->rows = rows;
+    a->cols_w = uint64_t(cols) * w;
+    a->new_cols_w = uint64_t(new_cols) * w;
+    a->words_per_elem = uint32_t(w);
+    a->pad = pad;
+    std::memset(a->fill, 0, sizeof(a->fill));
+    return DS_SUCCESS;
+}
+
+ds_status run_regular(const ds::RegArgs& a, cudaStream_t s) {
+    // No-ops: nothing moves and no fill cell exists / nothing is kept.
+    if (a.rows == 0 || a.cols_w == a.new_cols_w || a.new_cols_w == 0) return DS_SUCCESS;
+    std::lock_guard<std::mutex> lock(g_mu);
+    ds::Workspace* ws = nullptr;
+    ds_status st = get_workspace(ds::regular_tiles(a), s, &ws);
+    if (st != DS_SUCCESS) return st;
+    cudaError_t e = ds::launch_regular(a, *ws, s);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "regular kernel launch");
+}
+
+ds_status sync_default() {
+    cudaError_t e = cudaStreamSynchronize(nullptr);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "cudaStreamSynchronize");
+}
+
+}  // namespace
+
+namespace ds {
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+}  // namespace ds
+
+extern "C" {
+
+ds_status ds_pad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes,
+                    const void* fill, ds_stream_t stream) {
+    ds::RegArgs a{};
+    ds_status st = check_regular(ptr, rows, cols, new_cols, elem_bytes, true, &a);
+    if (st != DS_SUCCESS) return st;
+    if (fill) std::memcpy(a.fill, fill, elem_bytes);
+    return run_regular(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_unpad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes,
+                      ds_stream_t stream) {
+    ds::RegArgs a{};
+    ds_status st = check_regular(ptr, rows, cols, new_cols, elem_bytes, false, &a);
+    if (st != DS_SUCCESS) return st;
+    return run_regular(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_pad(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes) {
+    ds_status st = ds_pad_ex(ptr, rows, cols, new_cols, elem_bytes, nullptr, nullptr);
+    return st == DS_SUCCESS ? sync_default() : st;
+}
+
+ds_status ds_unpad(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes) {
+    ds_status st = ds_unpad_ex(ptr, rows, cols, new_cols, elem_bytes, nullptr);
+    return st == DS_SUCCESS ? sync_default() : st;
+}
+
+ds_status ds_compact_ex(void* ptr, size_t n, uint32_t remove_value, uint64_t* d_out_n,
+                        ds_stream_t stream) {
+    ds_status st = check_irregular(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Compact, 0, remove_value,
+                    nullptr, 0, d_out_n};
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_select_ex(void* ptr, size_t n, int predicate_id, uint32_t param, uint64_t* d_out_n,
+                       ds_stream_t stream) {
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Select, predicate_id, param,
+                    nullptr, 0, d_out_n};
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_unique_ex(void* ptr, size_t n, const uint64_t* d_halo, size_t halo_len,
+                       uint64_t* d_out_n, ds_stream_t stream) {
+    if (halo_len > 0 && d_halo == nullptr) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(d_halo, 8)) return DS_ERROR_INVALID_VALUE;
+    if (halo_len > 0xFFFFFFFFull) return DS_ERROR_UNSUPPORTED;
+    ds_status st = check_irregular(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Unique, 0, 0u,
+                    d_halo, halo_len, d_out_n};
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_compact(void* ptr, size_t n, uint32_t remove_value, size_t* out_n) {
+    if (!out_n) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(ptr, n, nullptr);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Compact, 0, remove_value,
+                    nullptr, 0, nullptr};
+    return irregular_blocking(a, out_n);
+}
+
+ds_status ds_select(void* ptr, size_t n, int predicate_id, size_t* out_n) {
+    if (!out_n) return DS_ERROR_INVALID_VALUE;
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(ptr, n, nullptr);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Select, predicate_id, 0u,
+                    nullptr, 0, nullptr};
+    return irregular_blocking(a, out_n);
+}
+
+ds_status ds_unique(void* ptr, size_t n, size_t* out_n) {
+    if (!out_n) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(ptr, n, nullptr);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Unique, 0, 0u, nullptr, 0, nullptr};
+    return irregular_blocking(a, out_n);
+}
+
+ds_status ds_halo_entry(const void* ptr, size_t n, uint64_t* d_entry, ds_stream_t stream) {
+    if (!d_entry || misaligned(d_entry, 8)) return DS_ERROR_INVALID_VALUE;
+    if (n > 0 && (ptr == nullptr || misaligned(ptr, 4))) return DS_ERROR_INVALID_VALUE;
+    cudaError_t e = ds::launch_halo_entry(static_cast<const uint32_t*>(ptr), n, d_entry,
+                                          reinterpret_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "halo entry launch");
+}
+
+ds_status ds_shard_offsets(const uint64_t* d_counts, size_t world, size_t rank, uint64_t* d_result,
+                           ds_stream_t stream) {
+    if (!d_counts || !d_result || world == 0 || rank >= world) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(d_counts, 8) || misaligned(d_result, 8)) return DS_ERROR_INVALID_VALUE;
+    if (world > 0xFFFFFFFFull) return DS_ERROR_UNSUPPORTED;
+    cudaError_t e = ds::launch_shard_offsets(d_counts, world, rank, d_result,
+                                             reinterpret_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "shard offsets launch");
+}
+
+const char* ds_status_string(ds_status s) {
+    switch (s) {
+    case DS_SUCCESS: return "DS_SUCCESS";
+    case DS_ERROR_INVALID_VALUE: return "DS_ERROR_INVALID_VALUE";
+    case DS_ERROR_UNSUPPORTED: return "DS_ERROR_UNSUPPORTED";
+    case DS_ERROR_OUT_OF_MEMORY: return "DS_ERROR_OUT_OF_MEMORY";
+    case DS_ERROR_CUDA: return "DS_ERROR_CUDA";
+    }
+    return "DS_ERROR_UNKNOWN";
+}
+
+const char* ds_last_error(void) { return g_err.c_str(); }
+
+ds_status ds_release_workspaces(void) {
+    std::lock_guard<std::mutex> lock(g_mu);
+    int cur = 0;
+    cudaGetDevice(&cur);
+    ds_status st = DS_SUCCESS;
+    for (auto& kv : g_ws) {
+        ds::Workspace& ws = kv.second;
+        if (cudaSetDevice(kv.first.first) != cudaSuccess) continue;
+        cudaDeviceSynchronize();
+        if (ws.status) cudaFree(ws.status);
+        if (ws.ctrl) cudaFree(ws.ctrl);
+        if (ws.h_count) cudaFreeHost(ws.h_count);
+    }
+    g_ws.clear();
+    cudaSetDevice(cur);
+    return st;
+}
+
+uint64_t ds_launch_count(void) { return g_launches.load(); }
+
+int ds_version(void) { return 100; }
+
+}  // extern "C"

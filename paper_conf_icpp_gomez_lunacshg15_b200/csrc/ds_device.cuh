@@ -1,0 +1,131 @@
+// ds_device.cuh -- device building blocks shared by the DS kernels (sm_100a).
+//
+//  * Dynamic tile ID allocation (the paper's Fig. 4) fused with a
+//    per-launch epoch: one 64-bit word {epoch:32 | ticket:32}.  The CTA that
+//    draws the LAST ticket of a launch re-arms the word for the next launch
+//    (epoch+1, ticket 0) -- every ticket of this launch has been drawn by
+//    then, so no memset launch is needed between calls.
+//  * Tile status words (the paper's per-WG flags, Fig. 3 P:92-103 / Fig. 7
+//    P:143-156) as 64-bit {state:2 | epoch:26 | count:36}.  A status whose
+//    epoch differs from the launch's is "not yet published" (R8: a zero
+//    count is never confused with "not ready").
+//  * Release/acquire at GPU scope (R10): publish with st.release.gpu after
+//    the tile's loads; poll with ld.relaxed.gpu (no L1 invalidation per
+//    poll) and execute ONE fence.acq_rel.gpu once every awaited status is
+//    seen.
+//  * 128-bit streaming loads/stores that do not allocate in L1.
+#pragma once
+
+#include <cstdint>
+
+namespace ds {
+
+constexpr uint64_t kStateShift = 62;
+constexpr uint64_t kEpochShift = 36;
+constexpr uint64_t kEpochMask = (1ull << 26) - 1;
+constexpr uint64_t kCountMask = (1ull << 36) - 1;
+constexpr uint64_t kStateAgg = 1;     // irregular: tile aggregate only
+constexpr uint64_t kStateLoaded = 1;  // regular: tile's sources are loaded
+constexpr uint64_t kStateIncl = 2;    // irregular: inclusive prefix known
+
+__host__ __device__ __forceinline__ uint64_t make_status(uint64_t state, uint64_t epoch,
+                                                         uint64_t count) {
+    return (state << kStateShift) | ((epoch & kEpochMask) << kEpochShift) | (count & kCountMask);
+}
+__device__ __forceinline__ uint32_t status_state(uint64_t s) { return uint32_t(s >> kStateShift); }
+__device__ __forceinline__ uint64_t status_count(uint64_t s) { return s & kCountMask; }
+__device__ __forceinline__ bool status_current(uint64_t s, uint64_t epoch) {
+    return status_state(s) != 0 && ((s >> kEpochShift) & kEpochMask) == (epoch & kEpochMask);
+}
+
+__device__ __forceinline__ uint64_t ld_relaxed_gpu(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_gpu(uint64_t* p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fence_acq_rel_gpu() {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+
+struct alignas(16) u32x4 {
+    uint32_t x, y, z, w;
+};
+
+__device__ __forceinline__ u32x4 ldg_stream_v4(const uint32_t* p) {
+    u32x4 r;
+    asm volatile("ld.global.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "l"(p));
+    return r;
+}
+__device__ __forceinline__ uint32_t ldg_stream(const uint32_t* p) {
+    uint32_t r;
+    asm volatile("ld.global.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    return r;
+}
+__device__ __forceinline__ void stg_stream_v4(uint32_t* p, uint32_t a, uint32_t b, uint32_t c,
+                                              uint32_t d) {
+    asm volatile("st.global.L1::no_allocate.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(a),
+                 "r"(b), "r"(c), "r"(d)
+                 : "memory");
+}
+__device__ __forceinline__ void stg_stream(uint32_t* p, uint32_t a) {
+    asm volatile("st.global.L1::no_allocate.u32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
+}
+
+// Fig. 4: thread 0 draws the dynamic tile id.  Returns
+// {tile, epoch}.  The CTA drawing ticket ntiles-1 re-arms the word.
+__device__ __forceinline__ void draw_ticket(uint64_t* ctrl, uint32_t ntiles, uint32_t& ticket,
+                                            uint32_t& epoch) {
+    unsigned long long old = atomicAdd(reinterpret_cast<unsigned long long*>(ctrl), 1ull);
+    ticket = uint32_t(old);
+    epoch = uint32_t(old >> 32);
+    if (ticket == ntiles - 1) {
+        uint32_t ne = epoch + 1;
+        if ((ne & kEpochMask) == 0) ne++;  // epoch 0 is never valid (zeroed status)
+        atomicExch(reinterpret_cast<unsigned long long*>(ctrl), (unsigned long long)ne << 32);
+    }
+}
+
+// Scheduling-stress hook (tests T3): with -DDS_DEBUG_DELAY the calling
+// thread sleeps a pseudo-random 0..4 us depending on (tile, site), which
+// reorders ticket -> load -> publish -> store across CTAs.  Compiled out of
+// the release library.
+__device__ __forceinline__ void debug_delay(uint64_t tile, uint32_t site) {
+#ifdef DS_DEBUG_DELAY
+    uint64_t z = tile * 0x9E3779B97F4A7C15ull + site * 0xBF58476D1CE4E5B9ull;
+    z ^= z >> 31;
+    z *= 0x94D049BB133111EBull;
+    z ^= z >> 29;
+    if ((z & 3) == 0) __nanosleep(uint32_t(z >> 40) % 4000u);
+#else
+    (void)tile;
+    (void)site;
+#endif
+}
+
+// Granlund-Montgomery round-up division by a runtime constant d (1 <= d <
+// 2^31), exact for every 32-bit numerator.
+struct FastDiv {
+    uint32_t d, mul, shift;
+};
+__host__ inline FastDiv make_fastdiv(uint32_t d) {
+    FastDiv f{d, 0, 0};
+    uint32_t l = 0;
+    while ((1ull << l) < d) ++l;
+    f.shift = l;
+    f.mul = uint32_t(((1ull << 32) * ((1ull << l) - d)) / d + 1);
+    return f;
+}
+__device__ __forceinline__ uint32_t fastdiv(uint32_t n, const FastDiv& f) {
+    uint64_t t = __umulhi(n, f.mul);
+    return uint32_t((t + n) >> f.shift);
+}
+
+}  // namespace ds

@@ -1,0 +1,58 @@
+// ds_internal.h -- host-side interface between the C ABI (ds_api.cu) and the
+// kernel launchers (ds_irregular.cu, ds_regular.cu, ds_shard.cu).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+
+namespace ds {
+
+// Per-(device, stream) workspace: tile status words + ticket/epoch word.
+struct Workspace {
+    uint64_t* status = nullptr;  // [cap_tiles]
+    size_t cap_tiles = 0;
+    uint64_t* ctrl = nullptr;    // {epoch:32 | ticket:32}; device_count follows
+    uint64_t* d_count = nullptr; // blocking forms' device-side out_n
+    uint64_t* h_count = nullptr; // pinned host mirror of d_count
+    uint64_t launches = 0;       // launches since the status array was zeroed
+};
+
+enum class IrregOp : int { Compact = 0, Select = 1, Unique = 2 };
+
+struct IrregArgs {
+    uint32_t* ptr;
+    size_t n;
+    IrregOp op;
+    int predicate;      // Select
+    uint32_t value;     // Compact: remove value; Select: param
+    const uint64_t* halo;  // Unique
+    size_t halo_len;
+    uint64_t* d_out_n;  // may be null
+};
+
+struct RegArgs {
+    uint32_t* ptr;
+    uint64_t rows;
+    uint64_t cols_w;      // words per row before
+    uint64_t new_cols_w;  // words per row after
+    uint32_t words_per_elem;
+    uint32_t fill[4];
+    bool pad;             // true: pad (expand, descending), false: unpad
+};
+
+// Tiles a launch of each kernel family needs (for workspace sizing).
+size_t irregular_tiles(const IrregArgs& a);
+size_t regular_tiles(const RegArgs& a);
+
+// Enqueue the kernels; return the cudaError_t of the launch.
+cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s);
+cudaError_t launch_regular(const RegArgs& a, Workspace& ws, cudaStream_t s);
+cudaError_t launch_halo_entry(const uint32_t* ptr, size_t n, uint64_t* d_entry, cudaStream_t s);
+cudaError_t launch_shard_offsets(const uint64_t* d_counts, size_t world, size_t rank,
+                                 uint64_t* d_result, cudaStream_t s);
+
+void count_launch();
+
+}  // namespace ds

@@ -1,0 +1,300 @@
+"""GPU parity (T2): libds CUDA kernels vs the CPU oracle, bit-exact on the
+WHOLE buffer including canary words around it (tolerance 0: integer /
+indexing work).  Inputs come from dsgen (seeded, shared by both sides).
+
+Sizes span several tiles (T = 4096 words) with ragged tails; pointers are
+misaligned by 0..3 words; fractions sweep 0..100 %.  Every call goes
+through the C ABI (ctypes binding)."""
+import numpy as np
+import pytest
+import torch
+
+import dsgen
+import oracle
+from gpu_util import DevBuf
+from paper_conf_icpp_gomez_lunacshg15_b200 import libds
+
+pytestmark = pytest.mark.gpu
+
+T = 4096
+SIZES = [1, 2, 3, 4, 5, 31, 32, 33, 1000, T - 1, T, T + 1, 2 * T - 1, 2 * T + 1, 3 * T + 7,
+         65537, 1_000_003]
+FRACS = [0.0, 0.1, 0.5, 0.9, 1.0]
+
+
+def _u32(t):
+    return t.numpy().view(np.uint32).copy()
+
+
+# ------------------------------------------------------------------ compaction
+@pytest.mark.parametrize("n", SIZES)
+@pytest.mark.parametrize("mis", [0, 1, 2, 3])
+def test_compact_sizes_misalignment(n, mis):
+    for k, f in enumerate(FRACS):
+        a = _u32(dsgen.compact_input(n, f, dsgen.seed_for(0, k + 7 * mis)))
+        buf = DevBuf(a, mis)
+        exp = buf.host_region()
+        m_exp = oracle.compact(exp, 0)
+        m = libds.ds_compact(buf.ptr, n, 0)
+        assert m == m_exp
+        buf.assert_equals(exp, f"compact n={n} mis={mis} f={f}")
+
+
+def _structured(n):
+    i = np.arange(n, dtype=np.uint32)
+    yield "all_removed_but_last", np.where(i == n - 1, i + 1, 0).astype(np.uint32)
+    yield "first_half_removed", np.where(i >= n // 2, i + 1, 0).astype(np.uint32)
+    yield "alternating", np.where(i % 2 == 1, i + 1, 0).astype(np.uint32)
+    yield "one_per_tile", np.where(i % T == T - 1, i + 1, 0).astype(np.uint32)
+    yield "odd_tiles_only", np.where((i // T) % 2 == 1, i + 1, 0).astype(np.uint32)
+    yield "runs_cross_tiles", np.where(((i + 1000) // 3000) % 2 == 0, i + 1, 0).astype(np.uint32)
+
+
+@pytest.mark.parametrize("n", [5 * T + 3, 200_000])
+def test_compact_structured_masks(n):
+    for name, a in _structured(n):
+        for mis in (0, 3):
+            buf = DevBuf(a, mis)
+            exp = buf.host_region()
+            m_exp = oracle.compact(exp, 0)
+            assert libds.ds_compact(buf.ptr, n, 0) == m_exp, name
+            buf.assert_equals(exp, name)
+
+
+def test_compact_remove_value_bitwise():
+    """R13: bitwise equality (-0.0 kept when removing +0.0; NaN removable)."""
+    f = np.array([0.0, -0.0, 1.5, np.nan, 0.0, np.nan] * 5000, dtype=np.float32)
+    a = f.view(np.uint32).copy()
+    for v in (0, int(a[3]), 0x80000000):
+        buf = DevBuf(a, 1)
+        exp = buf.host_region()
+        m_exp = oracle.compact(exp, v)
+        assert libds.ds_compact(buf.ptr, a.size, v) == m_exp
+        buf.assert_equals(exp, f"v={v:#x}")
+
+
+def test_compact_ex_stream_and_device_count():
+    n = 300_001
+    a = _u32(dsgen.compact_input(n, 0.37, 5))
+    buf = DevBuf(a, 2)
+    exp = buf.host_region()
+    m_exp = oracle.compact(exp, 0)
+    s = torch.cuda.Stream()
+    d_n = torch.full((1,), -1, dtype=torch.int64, device="cuda")
+    with torch.cuda.stream(s):
+        libds.ds_compact_ex(buf.ptr, n, 0, d_n, s)
+    s.synchronize()
+    assert int(d_n.item()) == m_exp
+    buf.assert_equals(exp, "ex")
+
+
+def test_compact_repeated_calls_same_stream():
+    """Epoch/ticket re-arming across back-to-back launches of different sizes."""
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    for rep in range(40):
+        n = [T * 3 + 1, 17, 100_000, 1][rep % 4] + rep
+        a = _u32(dsgen.compact_input(n, 0.5, 100 + rep))
+        buf = DevBuf(a, rep % 4)
+        exp = buf.host_region()
+        m_exp = oracle.compact(exp, 0)
+        libds.ds_compact_ex(buf.ptr, n, 0, d_n, None)
+        torch.cuda.synchronize()
+        assert int(d_n.item()) == m_exp
+        buf.assert_equals(exp, f"rep {rep}")
+
+
+def test_compact_repeat_race_hunt():
+    """Same medium input 200 times: any ordering bug shows up as a mismatch."""
+    n = 4_000_037
+    a = _u32(dsgen.compact_input(n, 0.5, 77))
+    exp = a.copy()
+    m_exp = oracle.compact(exp, 0)
+    src = torch.from_numpy(a.view(np.int32)).cuda()
+    work = torch.empty_like(src)
+    want = torch.from_numpy(exp.view(np.int32)).cuda()
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    for rep in range(200):
+        work.copy_(src)
+        libds.ds_compact_ex(work, n, 0, d_n, None)
+        assert int(d_n.item()) == m_exp, rep
+        assert torch.equal(work, want), rep
+
+
+# ---------------------------------------------------------------------- select
+PARAMS = [0, 1, 0x40490FDB, 0xC0000000, 0x7FFFFFFF, 0x7FC00000]
+
+
+@pytest.mark.parametrize("pred", range(libds.DS_PRED_COUNT))
+@pytest.mark.parametrize("n", [1, 33, T + 1, 3 * T + 7, 250_001])
+def test_select_predicates(pred, n):
+    a = _u32(dsgen.random_words(n, 1000 + pred + n))
+    specials = np.array([0, 0x80000000, 0x7FC00000, 0xFFC00001, 0x7F800000, 0xFF800000,
+                         0xFFFFFFFF, 1, 2, 0x00000003, 0x80000001], dtype=np.uint32)
+    a[::13] = np.resize(specials, a[::13].size)
+    for j, param in enumerate(PARAMS):
+        buf = DevBuf(a, (j + n) % 4)
+        exp = buf.host_region()
+        m_exp = oracle.select(exp, pred, param)
+        d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+        libds.ds_select_ex(buf.ptr, n, pred, param, d_n, None)
+        torch.cuda.synchronize()
+        assert int(d_n.item()) == m_exp, (pred, hex(param))
+        buf.assert_equals(exp, f"select pred={pred} param={param:#x}")
+
+
+def test_select_blocking_param_zero():
+    a = _u32(dsgen.random_words(77_777, 3))
+    for pred in range(libds.DS_PRED_COUNT):
+        buf = DevBuf(a, 1)
+        exp = buf.host_region()
+        m_exp = oracle.select(exp, pred, 0)
+        assert libds.ds_select(buf.ptr, a.size, pred) == m_exp
+        buf.assert_equals(exp, f"pred {pred}")
+
+
+@pytest.mark.parametrize("f", [i / 10 for i in range(11)])
+def test_select_threshold_sweep(f):
+    n = 1 << 20
+    a = _u32(dsgen.select_input(n, dsgen.seed_for(2, int(f * 10))))
+    t = dsgen.select_threshold(f) & 0xFFFFFFFF
+    buf = DevBuf(a, 0)
+    exp = buf.host_region()
+    m_exp = oracle.select(exp, libds.DS_PRED_I32_GT, t)
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    libds.ds_select_ex(buf.ptr, n, libds.DS_PRED_I32_GT, t, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == m_exp
+    buf.assert_equals(exp, f"f={f}")
+
+
+# ---------------------------------------------------------------------- unique
+@pytest.mark.parametrize("n", SIZES)
+@pytest.mark.parametrize("mis", [0, 3])
+def test_unique_runs_and_small_alphabets(n, mis):
+    cases = [("runs%.1f" % f, _u32(dsgen.unique_runs_input(n, f, 31 + k)))
+             for k, f in enumerate(FRACS)]
+    cases += [("bits1", _u32(dsgen.random_words(n, 5, bits=1))),
+              ("bits2", _u32(dsgen.random_words(n, 6, bits=2))),
+              ("hashed", _u32(dsgen.unique_hashed_input(n, 0.5, 7)))]
+    for name, a in cases:
+        buf = DevBuf(a, mis)
+        exp = buf.host_region()
+        m_exp = oracle.unique(exp)
+        assert libds.ds_unique(buf.ptr, n) == m_exp, name
+        buf.assert_equals(exp, f"unique {name} n={n} mis={mis}")
+
+
+def test_unique_tile_boundary_runs():
+    """Runs that end exactly at / straddle tile boundaries (P:280 boundary read)."""
+    n = 8 * T
+    i = np.arange(n)
+    for period in (T, T // 2, T + 1, 3, 1):
+        a = (i // period).astype(np.uint32)
+        for mis in range(4):
+            buf = DevBuf(a, mis)
+            exp = buf.host_region()
+            m_exp = oracle.unique(exp)
+            assert libds.ds_unique(buf.ptr, n) == m_exp
+            buf.assert_equals(exp, f"period {period} mis {mis}")
+
+
+def test_unique_halo():
+    """ds_unique_ex with a halo of earlier shards (R18): nearest non-empty wins."""
+    a = np.array([5, 5, 6, 6, 7], dtype=np.uint32)
+    cases = [([], None), ([(1 << 32) | 5], 5), ([(1 << 32) | 4], 4),
+             ([(1 << 32) | 5, 0], 5), ([(1 << 32) | 9, (1 << 32) | 5, 0, 0], 5), ([0, 0], None)]
+    for halo, prev in cases:
+        buf = DevBuf(a, 1)
+        exp = buf.host_region()
+        m_exp = oracle.unique(exp, prev=prev)
+        d_halo = torch.tensor(halo if halo else [0], dtype=torch.int64, device="cuda")
+        d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+        libds.ds_unique_ex(buf.ptr, a.size, d_halo if halo else None, len(halo), d_n, None)
+        torch.cuda.synchronize()
+        assert int(d_n.item()) == m_exp, halo
+        buf.assert_equals(exp, f"halo {halo}")
+
+
+# ------------------------------------------------------------------ pad / unpad
+def _pad_case(R, C, NC, eb, mis, fill=None, kind="index"):
+    w = eb // 4
+    a = _u32(dsgen.matrix_input(R, C, NC, eb, kind=kind))
+    buf = DevBuf(a, mis, capacity=a.size)
+    exp = buf.host_region()
+    fb = None if fill is None else np.asarray(fill, dtype=np.uint32).tobytes()
+    oracle.pad(exp, R, C, NC, eb, fb)
+    if fill is None:
+        libds.ds_pad(buf.ptr, R, C, NC, eb)
+    else:
+        libds.ds_pad_ex(buf.ptr, R, C, NC, eb, fb, None)
+    buf.assert_equals(exp, f"pad R={R} C={C} NC={NC} eb={eb} mis={mis}")
+    # and back (round trip; unpad leaves the tail as the padded buffer had it)
+    back = exp.copy()
+    oracle.unpad(back, R, NC, C, eb)
+    libds.ds_unpad(buf.ptr, R, NC, C, eb)
+    buf.assert_equals(back, f"unpad R={R} C={NC} NC={C} eb={eb} mis={mis}")
+    assert np.array_equal(back[:R * C * w], a[:R * C * w])
+
+
+def test_pad_unpad_brute_force_small():
+    for eb in (4, 8, 16):
+        w = eb // 4
+        fill = [0xF1F1F100 + j for j in range(w)]
+        for R in range(1, 5):
+            for C in range(0, 6):
+                for NC in range(C, 8):
+                    _pad_case(R, C, NC, eb, (R + C + NC) % 4, fill)
+
+
+@pytest.mark.parametrize("shape", [
+    (4000, 3990, 4000, 4),      # C2
+    (5000, 4900, 5000, 4),      # Fig. 2 / Fig. 8(c,d) shape
+    (1000, 1, 4100, 4),         # tiny rows, huge padding: wide windows
+    (3, 1_000_000, 1_000_001, 4),
+    (1, 1, 100_000, 4),
+    (100_000, 1, 3, 4),
+    (777, 1023, 1025, 8),
+    (333, 257, 300, 16),
+    (64, 4096, 8192, 4),
+    (4096, 1, 2, 4),
+])
+@pytest.mark.parametrize("mis", [0, 1])
+def test_pad_unpad_shapes(shape, mis):
+    R, C, NC, eb = shape
+    _pad_case(R, C, NC, eb, mis, fill=[0xABCD0000 + j for j in range(eb // 4)])
+
+
+def test_pad_c2_f32_values():
+    _pad_case(4000, 3990, 4000, 4, 0, kind="f32")
+
+
+@pytest.mark.parametrize("shape", [(10_000, 5000, 3, 4), (2000, 100_000, 10, 4), (50, 20_000, 19_000, 4),
+                                   (5, 3, 1, 16)])
+def test_unpad_large_drop_slow_path(shape):
+    R, C, NC, eb = shape
+    a = _u32(dsgen.matrix_input(R, C, NC, eb))
+    for mis in (0, 2):
+        buf = DevBuf(a, mis)
+        exp = buf.host_region()
+        oracle.unpad(exp, R, C, NC, eb)
+        libds.ds_unpad(buf.ptr, R, C, NC, eb)
+        buf.assert_equals(exp, f"unpad {shape} mis={mis}")
+
+
+def test_pad_table1_shape():
+    """Table I shape: 12000 x 11999 -> 12000, u32 index values."""
+    _pad_case(12000, 11999, 12000, 4, 0)
+
+
+def test_pad_repeat_race_hunt():
+    R, C, NC = 2000, 1999, 2003
+    a = _u32(dsgen.matrix_input(R, C, NC, 4))
+    exp = a.copy()
+    oracle.pad(exp, R, C, NC, 4)
+    src = torch.from_numpy(a.view(np.int32)).cuda()
+    want = torch.from_numpy(exp.view(np.int32)).cuda()
+    work = torch.empty_like(src)
+    for rep in range(100):
+        work.copy_(src)
+        libds.ds_pad_ex(work, R, C, NC, 4, None, None)
+        assert torch.equal(work, want), rep
