@@ -79,18 +79,73 @@ __device__ __forceinline__ void stg_stream(uint32_t* p, uint32_t a) {
     asm volatile("st.global.L1::no_allocate.u32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
 }
 
-// Fig. 4: thread 0 draws the dynamic tile id.  Returns
-// {tile, epoch}.  The CTA drawing ticket ntiles-1 re-arms the word.
-__device__ __forceinline__ void draw_ticket(uint64_t* ctrl, uint32_t ntiles, uint32_t& ticket,
+// Fig. 4: thread 0 draws the next dynamic tile id.  Returns
+// {ticket, epoch}.  A launch makes exactly `draws` draws in total (the
+// persistent kernels: ntiles + gridDim.x, every CTA's last draw fails); the
+// CTA that makes the final draw re-arms the word for the next launch.
+__device__ __forceinline__ void draw_ticket(uint64_t* ctrl, uint32_t draws, uint32_t& ticket,
                                             uint32_t& epoch) {
     unsigned long long old = atomicAdd(reinterpret_cast<unsigned long long*>(ctrl), 1ull);
     ticket = uint32_t(old);
     epoch = uint32_t(old >> 32);
-    if (ticket == ntiles - 1) {
+    if (ticket == draws - 1) {
         uint32_t ne = epoch + 1;
         if ((ne & kEpochMask) == 0) ne++;  // epoch 0 is never valid (zeroed status)
         atomicExch(reinterpret_cast<unsigned long long*>(ctrl), (unsigned long long)ne << 32);
     }
+}
+
+// ---- shared-memory mbarrier + 1-D TMA bulk copy (cp.async.bulk) --------
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_fence_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred P;\n"
+        "DS_WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
+        "@!P bra DS_WAIT_%=;\n"
+        "}\n" ::"r"(smem_addr(bar)),
+        "r"(parity)
+        : "memory");
+}
+// Named barrier among `count` threads (a subset of the CTA, whole warps).
+__device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t count) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+
+// Global -> shared bulk copy of `bytes` (multiple of 16, both addresses
+// 16-byte aligned), completing on `bar`.  Streams through L2 (evict-first).
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "{\n"
+        ".reg .b64 pol;\n"
+        "createpolicy.fractional.L2::evict_first.b64 pol, 1.0;\n"
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1], %2, [%3], pol;\n"
+        "}\n" ::"r"(smem_addr(dst)),
+        "l"(src), "r"(bytes), "r"(smem_addr(bar))
+        : "memory");
 }
 
 // Scheduling-stress hook (tests T3): with -DDS_DEBUG_DELAY the calling
@@ -126,6 +181,29 @@ __host__ inline FastDiv make_fastdiv(uint32_t d) {
 __device__ __forceinline__ uint32_t fastdiv(uint32_t n, const FastDiv& f) {
     uint64_t t = __umulhi(n, f.mul);
     return uint32_t((t + n) >> f.shift);
+}
+
+// Same for 64-bit numerators (d < 2^32): q = (t + ((n - t) >> 1)) >> (l-1),
+// t = mulhi64(n, m), m = floor(2^64 (2^l - d) / d) + 1.  Exact for all n.
+struct FastDiv64 {
+    uint64_t d, mul;
+    uint32_t shift;
+};
+__host__ inline FastDiv64 make_fastdiv64(uint64_t d) {
+    FastDiv64 f{d, 0, 0};
+    uint32_t l = 0;
+    while ((1ull << l) < d) ++l;
+    f.shift = l;
+    if (l > 0) {
+        unsigned __int128 num = (unsigned __int128)((1ull << l) - d) << 64;
+        f.mul = uint64_t(num / d) + 1;
+    }
+    return f;
+}
+__device__ __forceinline__ uint64_t fastdiv64(uint64_t n, const FastDiv64& f) {
+    if (f.shift == 0) return n;  // d == 1
+    const uint64_t t = __umul64hi(n, f.mul);
+    return (t + ((n - t) >> 1)) >> (f.shift - 1);
 }
 
 }  // namespace ds

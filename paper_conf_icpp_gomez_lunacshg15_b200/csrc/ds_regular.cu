@@ -5,7 +5,11 @@
 // The matrix is handled as 32-bit words: an element of elem_bytes is
 // elem_bytes/4 consecutive words, so a row of C elements is Cw = C*eb/4
 // words.  One CTA = one OUTPUT tile of T = THREADS*ITEMS words (the paper's
-// work-groups are "oblivious to number of rows and row boundaries"):
+// work-groups are "oblivious to number of rows and row boundaries").
+// Persistent CTAs double-buffer their tiles' sources in shared memory: once
+// a tile's LOADED status is published the CTA draws the next tile and
+// streams its source span in through one TMA bulk copy while the current
+// tile is gathered and stored.  Per tile:
 //   r1 ticket + direction   pad expands (src(q) <= q): tiles in DESCENDING
 //                           order; unpad shrinks (src(q) >= q): ASCENDING
 //                           ("a sequential order (ascendant or descendant)",
@@ -31,41 +35,50 @@
 namespace ds {
 namespace {
 
+constexpr int64_t kNoTile = -1;
+
 struct RegParams {
     uint32_t* abase;  // 16-byte-aligned base; virtual word 0
     uint64_t mis;     // ptr - abase in words
     uint64_t out_words, in_words;
     uint32_t Cw, NCw;
     FastDiv div_nc;
+    FastDiv64 div_nc64, div_c64;
     uint32_t fill[4];
     uint32_t wmask;   // words_per_elem - 1
     uint32_t ntiles;
+    uint32_t draws;   // ntiles + gridDim.x
     uint64_t* status;
     uint64_t* ctrl;
 };
 
 struct TileGeom {
+    int64_t k;            // tile index (kNoTile: none)
     int64_t q0, q1;       // output words [q0, q1) of this tile
     int64_t row0;         // row of q0
-    uint32_t col0;        // column (word) of q0
     int64_t slo;          // first source word (input index) of the tile's data cells
     int64_t span;         // number of source words [slo, slo+span)
     int64_t sb;           // 16-byte aligned virtual start of the staged span
     int64_t win_lo, win_hi;  // tiles to wait for (inclusive); empty if lo > hi
+    uint32_t col0;        // column (word) of q0
     int32_t base_rel;     // row0*Cw - slo
     int32_t fast;         // staged span fits in shared memory
+    uint32_t bytes;       // bulk copy size (fast path)
 };
 
-template <bool PAD, int T, int SPAN_CAP>
+// Closed-form tile geometry.  Only 64-bit divisions by the
+// two row lengths, done with multiply-high (FastDiv64).
+template <bool PAD, int T, int STAGE>
 __device__ void tile_geometry(const RegParams& p, int64_t k, TileGeom& g) {
     const int64_t Cw = p.Cw, NCw = p.NCw, mis = int64_t(p.mis);
     const int64_t V0 = k * T;
+    g.k = k;
     g.q0 = V0 - mis > 0 ? V0 - mis : 0;
     g.q1 = V0 + T - mis < int64_t(p.out_words) ? V0 + T - mis : int64_t(p.out_words);
-    g.row0 = g.q0 / NCw;
+    g.row0 = int64_t(fastdiv64(uint64_t(g.q0), p.div_nc64));
     g.col0 = uint32_t(g.q0 - g.row0 * NCw);
     const int64_t last = g.q1 - 1;
-    const int64_t row1 = last / NCw;
+    const int64_t row1 = int64_t(fastdiv64(uint64_t(last), p.div_nc64));
     const int64_t col1 = last - row1 * NCw;
     int64_t slo, shi;
     if (PAD) {
@@ -78,7 +91,9 @@ __device__ void tile_geometry(const RegParams& p, int64_t k, TileGeom& g) {
     g.slo = slo;
     g.span = shi >= slo ? shi - slo + 1 : 0;
     g.sb = (slo + mis) & ~int64_t(3);
-    g.fast = (slo + mis + g.span - g.sb) <= SPAN_CAP;
+    const int64_t se = (slo + mis + g.span + 3) & ~int64_t(3);  // may pass the end by <= 3 words
+    g.fast = (se - g.sb) <= STAGE;
+    g.bytes = g.span > 0 && g.fast ? uint32_t(se - g.sb) * 4u : 0u;
     g.base_rel = int32_t(g.row0 * Cw - slo);
 
     // Sources physically inside this tile's output range: input words [P0, P1).
@@ -87,15 +102,15 @@ __device__ void tile_geometry(const RegParams& p, int64_t k, TileGeom& g) {
     g.win_lo = 1;
     g.win_hi = 0;
     if (P0 < P1) {
+        const int64_t r = int64_t(fastdiv64(uint64_t(P0), p.div_c64)), c = P0 - r * Cw;
+        const int64_t r2 = int64_t(fastdiv64(uint64_t(P1 - 1), p.div_c64)), c2 = (P1 - 1) - r2 * Cw;
         if (PAD) {  // every input word is kept; out(p) = p + row(p)*(NCw-Cw) >= p
-            const int64_t olo = P0 + (P0 / Cw) * (NCw - Cw);
-            const int64_t ohi = (P1 - 1) + ((P1 - 1) / Cw) * (NCw - Cw);
+            const int64_t olo = P0 + r * (NCw - Cw);
+            const int64_t ohi = (P1 - 1) + r2 * (NCw - Cw);
             const int64_t wl = (olo + mis) / T, wh = (ohi + mis) / T;
             g.win_lo = wl > k + 1 ? wl : k + 1;
             g.win_hi = wh;
         } else {    // only columns < NCw are read; out(p) = row*NCw + col <= p
-            const int64_t r = P0 / Cw, c = P0 - r * Cw;
-            const int64_t r2 = (P1 - 1) / Cw, c2 = (P1 - 1) - r2 * Cw;
             // first / last kept source word in [P0, P1) and their outputs
             const int64_t pf = c < NCw ? P0 : (r + 1) * Cw;
             const int64_t pl = c2 < NCw ? P1 - 1 : r2 * Cw + NCw - 1;
@@ -124,10 +139,10 @@ __device__ __forceinline__ void wait_loaded(const uint64_t* __restrict__ status,
     for (int64_t base = lo; base <= hi; base += 32) {
         const int64_t idx = base + lane;
         bool ok = idx > hi || status_current(ld_relaxed_gpu(status + idx), epoch);
-        uint32_t ns = 8;
+        uint32_t ns = 32;
         while (!__all_sync(0xffffffffu, ok)) {
             __nanosleep(ns);
-            ns = ns < 256 ? ns * 2 : 256;
+            ns = ns < 512 ? ns * 2 : 512;
             if (!ok) ok = status_current(ld_relaxed_gpu(status + idx), epoch);
         }
     }
@@ -135,153 +150,225 @@ __device__ __forceinline__ void wait_loaded(const uint64_t* __restrict__ status,
     __syncwarp();
 }
 
-template <int THREADS, int ITEMS, bool PAD>
-__global__ void __launch_bounds__(THREADS) regular_kernel(const RegParams p) {
-    constexpr int VEC = ITEMS / 4;
-    constexpr int T = THREADS * ITEMS;
-    constexpr int SPAN_CAP = T + 512;
-    constexpr int LOAD_ITERS = (SPAN_CAP / 4 + THREADS - 1) / THREADS;
+constexpr int kConsumerWarps = 8;
+constexpr int kCT = 32 * kConsumerWarps;  // consumer threads
+constexpr int kItems = 32;                // output words per consumer thread
+constexpr int kVec = kItems / 4;
+constexpr int kT = kCT * kItems;          // 8192 output words = 32 KB per tile
+constexpr int kStageWords = kT + 512;     // staged source span cap (words)
+constexpr int kStages = 3;
+constexpr int kThreads = 32 * (1 + kConsumerWarps);
+constexpr size_t kSmem = size_t(kStages) * kStageWords * 4;
 
-    __shared__ alignas(16) uint32_t s_src[SPAN_CAP];
-    __shared__ TileGeom s_g;
-    __shared__ uint32_t s_epoch;
-    __shared__ int64_t s_k;
+struct StageMeta {
+    TileGeom g;
+    uint32_t epoch;
+};
+
+// Producer, slow path (the source span does not fit a stage: unpad dropping
+// many columns of short rows): the warp gathers the tile's source words
+// directly, stored in OUTPUT order.
+template <bool PAD>
+__device__ void gather_slow(const RegParams& p, const TileGeom& g, uint32_t* stage, int lane) {
+    const int64_t mis = int64_t(p.mis);
+    const uint32_t cnt = uint32_t(g.q1 - g.q0);
+    for (uint32_t x0 = 0; x0 < cnt; x0 += 32 * 8) {
+        uint32_t val[8];
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const uint32_t x = x0 + 32 * u + lane;
+            val[u] = 0;
+            if (x < cnt) {
+                const uint32_t t = g.col0 + x;
+                const uint32_t dr = fastdiv(t, p.div_nc);
+                const uint32_t col = t - dr * p.NCw;
+                if (PAD && col >= p.Cw) val[u] = fill_word(p, col);
+                else val[u] = ldg_stream(p.abase + (g.row0 + dr) * int64_t(p.Cw) + col + mis);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+            const uint32_t x = x0 + 32 * u + lane;
+            if (x < cnt) stage[x] = val[u];
+        }
+    }
+    __syncwarp();
+}
+
+template <bool PAD>
+__global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p) {
+    extern __shared__ __align__(128) uint32_t smem[];
+    __shared__ __align__(8) uint64_t bar_full[kStages], bar_loaded[kStages], bar_empty[kStages];
+    __shared__ StageMeta meta[kStages];
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid == 0) {  // r1
-        uint32_t t, e;
-        draw_ticket(p.ctrl, p.ntiles, t, e);
-        const int64_t k = PAD ? int64_t(p.ntiles) - 1 - t : int64_t(t);
-        s_k = k;
-        s_epoch = e;
-        tile_geometry<PAD, T, SPAN_CAP>(p, k, s_g);
-        debug_delay(uint64_t(k), 0);
+    if (tid == 0) {
+        for (int s = 0; s < kStages; ++s) {
+            mbar_init(&bar_full[s], 1);
+            mbar_init(&bar_loaded[s], 1);
+            mbar_init(&bar_empty[s], kConsumerWarps);
+        }
+        mbar_fence_init();
     }
     __syncthreads();
-    const int64_t k = s_k;
-    const uint32_t epoch = s_epoch;
-    const TileGeom g = s_g;
     const int64_t mis = int64_t(p.mis);
-    const int64_t V0 = k * T;
 
-    // r2: load stage.
-    if (g.span > 0) {
-        const int64_t vlo = g.slo + mis, vhi = g.slo + mis + g.span;  // virtual [vlo, vhi)
-        if (g.fast) {
-            u32x4 r[LOAD_ITERS];
-#pragma unroll
-            for (int it = 0; it < LOAD_ITERS; ++it) {
-                const int64_t u = g.sb + 4 * int64_t(it * THREADS + tid);
-                if (u >= vlo && u + 4 <= vhi) {
-                    r[it] = ldg_stream_v4(p.abase + u);
-                } else if (u < vhi) {
-                    uint32_t w[4];
-#pragma unroll
-                    for (int kk = 0; kk < 4; ++kk) {
-                        const int64_t e = u + kk;
-                        w[kk] = (e >= vlo && e < vhi) ? ldg_stream(p.abase + e) : 0u;
-                    }
-                    r[it] = u32x4{w[0], w[1], w[2], w[3]};
+    if (warp == 0) {
+        // ------------------------------------------------ producer warp
+        // r1 draw, r2 load, r3a publish LOADED as soon as the sources landed.
+        for (uint32_t k = 0;; ++k) {
+            const int s = k % kStages;
+            const uint32_t use = k / kStages;
+            uint32_t* stage = smem + s * kStageWords;
+            mbar_wait(&bar_empty[s], (use & 1) ^ 1);  // consumers released tile k - kStages
+            uint32_t t = 0, epoch = 0;
+            if (lane == 0) draw_ticket(p.ctrl, p.draws, t, epoch);
+            t = __shfl_sync(0xffffffffu, t, 0);
+            epoch = __shfl_sync(0xffffffffu, epoch, 0);
+            if (t >= p.ntiles) {  // one failed draw per CTA ends its work
+                if (lane == 0) {
+                    meta[s].g.k = kNoTile;
+                    mbar_arrive(&bar_loaded[s]);
+                }
+                break;
+            }
+            const int64_t kt = PAD ? int64_t(p.ntiles) - 1 - t : int64_t(t);
+            if (lane == 0) {
+                debug_delay(uint64_t(kt), 0);
+                tile_geometry<PAD, kT, kStageWords>(p, kt, meta[s].g);
+                meta[s].epoch = epoch;
+                if (meta[s].g.bytes) {
+                    fence_proxy_async_smem();
+                    mbar_arrive_expect_tx(&bar_full[s], meta[s].g.bytes);
+                    bulk_g2s(stage, p.abase + meta[s].g.sb, meta[s].g.bytes, &bar_full[s]);
                 }
             }
-#pragma unroll
-            for (int it = 0; it < LOAD_ITERS; ++it) {
-                const int64_t u = g.sb + 4 * int64_t(it * THREADS + tid);
-                if (u < vhi) *reinterpret_cast<u32x4*>(s_src + 4 * (it * THREADS + tid)) = r[it];
+            __syncwarp();
+            const TileGeom& g = meta[s].g;
+            if (!g.bytes) {
+                // slow path, or no sources at all (all fill): complete the full
+                // barrier's phase by a plain arrival to keep its parity in step
+                if (g.span > 0) gather_slow<PAD>(p, g, stage, lane);
+                if (lane == 0) mbar_arrive(&bar_full[s]);
             }
-        } else {
-            // Span too long for shared memory (unpad dropping many columns of
-            // short rows): gather the tile's source words directly, staged in
-            // output order.
+            mbar_wait(&bar_full[s], use & 1);
+            if (lane == 0) {
+                debug_delay(uint64_t(kt), 1);
+                st_release_gpu(p.status + kt, make_status(kStateLoaded, epoch, 0));
+                mbar_arrive(&bar_loaded[s]);
+            }
+        }
+    } else {
+        // ------------------------------------------------ consumer warps
+        const int ct = tid - 32;
+        for (uint32_t k = 0;; ++k) {
+            const int s = k % kStages;
+            const uint32_t use = k / kStages;
+            const uint32_t* stage = smem + s * kStageWords;
+            mbar_wait(&bar_loaded[s], use & 1);
+            const TileGeom g = meta[s].g;
+            if (g.k == kNoTile) break;
+            const int64_t V0 = g.k * kT;
+
+            // r3b: the first consumer warp waits for the earlier-ticketed tiles
+            // whose sources lie in this tile's output range ...
+            if (warp == 1 && g.win_lo <= g.win_hi)
+                wait_loaded(p.status, g.win_lo, g.win_hi, meta[s].epoch, lane);
+
+            // ... while every consumer gathers its outputs (r4).
+            uint32_t o[kVec][4];
+            const int32_t soff = int32_t(g.slo + mis - g.sb);
 #pragma unroll
-            for (int i = 0; i < VEC; ++i) {
+            for (int i = 0; i < kVec; ++i) {
+                const int64_t vq = V0 + 4 * int64_t(i * kCT + ct) - mis;  // output word of slot 0
+                const int64_t xq = vq - g.q0;
+                uint32_t t = uint32_t(xq) + g.col0;  // only meaningful when vq >= q0
+                uint32_t dr = fastdiv(t, p.div_nc);
+                uint32_t col = t - dr * p.NCw;
 #pragma unroll
                 for (int kk = 0; kk < 4; ++kk) {
-                    const int64_t q = V0 + 4 * int64_t(i * THREADS + tid) + kk - mis;
-                    if (q < g.q0 || q >= g.q1) continue;
-                    const uint32_t x = uint32_t(q - g.q0);
-                    const uint32_t t = g.col0 + x;
-                    const uint32_t dr = fastdiv(t, p.div_nc);
-                    const uint32_t col = t - dr * p.NCw;
-                    uint32_t val;
-                    if (PAD && col >= p.Cw) val = fill_word(p, col);
-                    else val = ldg_stream(p.abase + (g.row0 + dr) * int64_t(p.Cw) + col + mis);
-                    s_src[x] = val;
+                    const int64_t q = vq + kk;
+                    uint32_t val = 0;
+                    if (q >= g.q0 && q < g.q1) {
+                        if (q == g.q0 && xq < 0) {  // tile 0 with a misaligned ptr
+                            dr = 0;
+                            col = g.col0;
+                        }
+                        if (!g.bytes && g.span > 0) {
+                            val = stage[uint32_t(q - g.q0)];  // slow path: output order
+                        } else if (PAD && col >= p.Cw) {
+                            val = fill_word(p, col);
+                        } else {
+                            const int32_t srel = g.base_rel + int32_t(dr * p.Cw + col);
+                            val = stage[srel + soff];
+                        }
+                    }
+                    o[i][kk] = val;
+                    if (++col == p.NCw) {
+                        col = 0;
+                        ++dr;
+                    }
                 }
             }
-        }
-    }
-    __syncthreads();  // the tile's loads are performed (values are in smem)
-    if (tid == 0) {
-        debug_delay(uint64_t(k), 1);
-        st_release_gpu(p.status + k, make_status(kStateLoaded, epoch, 0));
-    }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&bar_empty[s]);  // this warp is done with the stage
+            if (ct == 0) debug_delay(uint64_t(g.k), 2);
+            named_bar_sync(1, kCT);  // the window wait (acquire fence) precedes every store
 
-    // r3 (warp 0) overlapped with r4 (all warps).
-    if (warp == 0 && g.win_lo <= g.win_hi) wait_loaded(p.status, g.win_lo, g.win_hi, epoch, lane);
-
-    uint32_t o[VEC][4];
-    const int32_t soff = int32_t(g.slo + mis - g.sb);
+            // r5: store stage.
 #pragma unroll
-    for (int i = 0; i < VEC; ++i) {
-        const int64_t vq = V0 + 4 * int64_t(i * THREADS + tid) - mis;  // output word of slot 0
-        const int64_t xq = vq - g.q0;
-        uint32_t t = uint32_t(xq) + g.col0;  // only meaningful when vq >= q0
-        uint32_t dr = fastdiv(t, p.div_nc);
-        uint32_t col = t - dr * p.NCw;
-#pragma unroll
-        for (int kk = 0; kk < 4; ++kk) {
-            const int64_t q = vq + kk;
-            uint32_t val = 0;
-            if (q >= g.q0 && q < g.q1) {
-                if (q == g.q0 && xq < 0) {  // tile 0 with a misaligned ptr
-                    dr = 0;
-                    col = g.col0;
-                }
-                if (!g.fast && g.span > 0) {
-                    val = s_src[uint32_t(q - g.q0)];
-                } else if (PAD && col >= p.Cw) {
-                    val = fill_word(p, col);
+            for (int i = 0; i < kVec; ++i) {
+                const int64_t u = V0 + 4 * int64_t(i * kCT + ct);  // virtual
+                const int64_t q = u - mis;
+                if (q >= 0 && q + 4 <= int64_t(p.out_words)) {
+                    stg_stream_v4(p.abase + u, o[i][0], o[i][1], o[i][2], o[i][3]);
                 } else {
-                    const int32_t srel = g.base_rel + int32_t(dr * p.Cw + col);
-                    val = s_src[srel + soff];
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk)
+                        if (q + kk >= 0 && q + kk < int64_t(p.out_words))
+                            stg_stream(p.abase + u + kk, o[i][kk]);
                 }
             }
-            o[i][kk] = val;
-            if (++col == p.NCw) {
-                col = 0;
-                ++dr;
-            }
-        }
-    }
-    if (tid == 0) debug_delay(uint64_t(k), 2);
-    __syncthreads();  // warp 0's window wait (with its acquire fence) is done
-
-    // r5: store stage.
-#pragma unroll
-    for (int i = 0; i < VEC; ++i) {
-        const int64_t u = V0 + 4 * int64_t(i * THREADS + tid);  // virtual
-        const int64_t q = u - mis;
-        if (q >= 0 && q + 4 <= int64_t(p.out_words)) {
-            stg_stream_v4(p.abase + u, o[i][0], o[i][1], o[i][2], o[i][3]);
-        } else {
-#pragma unroll
-            for (int kk = 0; kk < 4; ++kk)
-                if (q + kk >= 0 && q + kk < int64_t(p.out_words)) stg_stream(p.abase + u + kk, o[i][kk]);
         }
     }
 }
 
-constexpr int kThreads = 256;
-constexpr int kItems = 16;
-constexpr int kTile = kThreads * kItems;
+struct LaunchCache {
+    int dev = -1, sms = 0, per_sm = 0;
+};
+
+template <bool PAD>
+cudaError_t launch_dir(RegParams p, cudaStream_t s) {
+    static thread_local LaunchCache lc;
+    auto kern = regular_kernel<PAD>;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (lc.dev != dev) {
+        if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(kSmem))) !=
+            cudaSuccess)
+            return e;
+        if ((e = cudaDeviceGetAttribute(&lc.sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
+            return e;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&lc.per_sm, kern, kThreads, kSmem)) !=
+            cudaSuccess)
+            return e;
+        if (lc.per_sm < 1) lc.per_sm = 1;
+        lc.dev = dev;
+    }
+    uint64_t grid = uint64_t(lc.sms) * lc.per_sm;
+    if (grid > p.ntiles) grid = p.ntiles;
+    p.draws = p.ntiles + uint32_t(grid);
+    kern<<<uint32_t(grid), kThreads, kSmem, s>>>(p);
+    return cudaGetLastError();
+}
 
 }  // namespace
 
 size_t regular_tiles(const RegArgs& a) {
     const uint64_t mis = (reinterpret_cast<uintptr_t>(a.ptr) >> 2) & 3u;
     const uint64_t out_words = a.rows * a.new_cols_w;
-    return size_t((out_words + mis + kTile - 1) / kTile);
+    return size_t((out_words + mis + kT - 1) / kT);
 }
 
 cudaError_t launch_regular(const RegArgs& a, Workspace& ws, cudaStream_t s) {
@@ -294,15 +381,15 @@ cudaError_t launch_regular(const RegArgs& a, Workspace& ws, cudaStream_t s) {
     p.Cw = uint32_t(a.cols_w);
     p.NCw = uint32_t(a.new_cols_w);
     p.div_nc = make_fastdiv(p.NCw);
+    p.div_nc64 = make_fastdiv64(p.NCw);
+    p.div_c64 = make_fastdiv64(p.Cw ? p.Cw : 1);
     for (int i = 0; i < 4; ++i) p.fill[i] = a.fill[i];
     p.wmask = a.words_per_elem - 1;
     p.ntiles = uint32_t(regular_tiles(a));
     p.status = ws.status;
     p.ctrl = ws.ctrl;
     count_launch();
-    if (a.pad) regular_kernel<kThreads, kItems, true><<<p.ntiles, kThreads, 0, s>>>(p);
-    else regular_kernel<kThreads, kItems, false><<<p.ntiles, kThreads, 0, s>>>(p);
-    return cudaGetLastError();
+    return a.pad ? launch_dir<true>(p, s) : launch_dir<false>(p, s);
 }
 
 }  // namespace ds

@@ -1,0 +1,20 @@
+"""T3: scheduling stress with the delay-injection build (libds_stress.so)."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+from paper_conf_icpp_gomez_lunacshg15_b200 import build
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+@pytest.mark.gpu
+def test_delay_injection_parity():
+    lib = build.build("stress")
+    env = dict(os.environ, LIBDS_PATH=lib)
+    r = subprocess.run([sys.executable, os.path.join(HERE, "stress_driver.py"), "12"],
+                       env=env, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    assert "stress OK" in r.stdout
