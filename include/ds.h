@@ -153,6 +153,14 @@ const char* ds_last_error(void);
 ds_status ds_release_workspaces(void);
 /* Number of kernel launches libds issued in this process (for bench.py). */
 uint64_t ds_launch_count(void);
+/* Diagnostics: while set, every DS kernel launch whose tile count fits
+ * `capacity_tiles` records 16 uint64 per tile into the DEVICE buffer d_trace
+ * (globaltimer ns: 0 drawn, 1 landed, 2 aggregate published, 3 look-back
+ * start, 4 prefix published, 5 stores start, 6 stores issued; 7 SM id;
+ * 8 look-back rounds, 9 polls, 10 first round read, 11 resolved, 12 after
+ * the acquire fence).
+ * NULL disables.  Development aid for DESIGN.md §7, not used by the API.  */
+ds_status ds_debug_set_trace(uint64_t* d_trace, size_t capacity_tiles);
 /* Library version, major*10000 + minor*100 + patch.                      */
 int ds_version(void);
 

@@ -7,6 +7,7 @@ paper_conf_icpp_gomez_lunacshg15_b200/lib/libds[<suffix>].so (a directory of
 its own so Python never mistakes it for an extension module).  Variants:
   release : -O3 -lineinfo                            -> libds.so
   stress  : -DDS_DEBUG_DELAY (random per-CTA delays) -> libds_stress.so
+  strict  : -DDS_STRICT_ORDER (release/acquire status ordering) -> libds_strict.so
 The CUDA runtime is linked statically so the library does not depend on
 which libcudart the host process (torch) has loaded.
 """
@@ -28,6 +29,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 VARIANTS = {
     "release": ("libds.so", []),
     "stress": ("libds_stress.so", ["-DDS_DEBUG_DELAY=1"]),
+    "strict": ("libds_strict.so", ["-DDS_STRICT_ORDER=1"]),
 }
 
 
@@ -51,12 +53,14 @@ def _newest_dep_mtime() -> float:
     return max(os.path.getmtime(d) for d in deps)
 
 
-def build(variant: str = "release", force: bool = False, verbose: bool = False) -> str:
-    out = lib_path(variant)
+def build(variant: str = "release", force: bool = False, verbose: bool = False,
+          extra_flags: list[str] | None = None, out_name: str | None = None) -> str:
+    """Build one variant; extra_flags/out_name build ad-hoc tuning variants."""
+    out = os.path.join(LIBDIR, out_name) if out_name else lib_path(variant)
     if not force and os.path.exists(out) and os.path.getmtime(out) >= _newest_dep_mtime():
         return out
-    extra = VARIANTS[variant][1]
-    objdir = os.path.join(ROOT, "build", variant)
+    extra = VARIANTS[variant][1] + list(extra_flags or [])
+    objdir = os.path.join(ROOT, "build", out_name.replace(".so", "") if out_name else variant)
     os.makedirs(objdir, exist_ok=True)
     os.makedirs(LIBDIR, exist_ok=True)
     common = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
@@ -87,8 +91,10 @@ def main() -> None:
     ap.add_argument("--force", action="store_true")
     ap.add_argument("--verbose", action="store_true")
     ap.add_argument("--variant", default="release", choices=sorted(VARIANTS))
+    ap.add_argument("-D", action="append", default=[], help="extra -D for a tuning build")
+    ap.add_argument("--out", default=None, help="library file name for a tuning build")
     a = ap.parse_args()
-    print(build(a.variant, a.force, a.verbose))
+    print(build(a.variant, a.force, a.verbose, [f"-D{d}" for d in a.D], a.out))
 
 
 if __name__ == "__main__":

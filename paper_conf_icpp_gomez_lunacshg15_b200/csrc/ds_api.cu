@@ -25,6 +25,8 @@ constexpr uint64_t kResetEvery = 1ull << 25;         // zero statuses before the
 std::mutex g_mu;
 std::map<std::pair<int, uintptr_t>, ds::Workspace> g_ws;
 std::atomic<uint64_t> g_launches{0};
+std::atomic<uint64_t*> g_trace{nullptr};
+std::atomic<size_t> g_trace_cap{0};
 thread_local std::string g_err;
 
 ds_status fail(cudaError_t e, const char* what) {
@@ -62,7 +64,7 @@ ds_status get_workspace(size_t tiles, cudaStream_t s, ds::Workspace** out) {
             ws.cap_tiles = 0;
         }
         size_t cap = tiles < 1024 ? 1024 : tiles;
-        if ((e = cudaMalloc(&ws.status, cap * sizeof(uint64_t))) != cudaSuccess) {
+        if ((e = cudaMalloc(&ws.status, cap * ds::kStatusStride * sizeof(uint64_t))) != cudaSuccess) {
             ws.status = nullptr;
             return e == cudaErrorMemoryAllocation ? DS_ERROR_OUT_OF_MEMORY : fail(e, "cudaMalloc");
         }
@@ -70,7 +72,8 @@ ds_status get_workspace(size_t tiles, cudaStream_t s, ds::Workspace** out) {
         ws.launches = kResetEvery;  // force the zeroing below
     }
     if (ws.launches >= kResetEvery) {
-        if ((e = cudaMemsetAsync(ws.status, 0, ws.cap_tiles * sizeof(uint64_t), s)) != cudaSuccess)
+        if ((e = cudaMemsetAsync(ws.status, 0, ws.cap_tiles * ds::kStatusStride * sizeof(uint64_t), s)) !=
+            cudaSuccess)
             return fail(e, "cudaMemsetAsync");
         ws.launches = 0;
     }
@@ -172,6 +175,7 @@ ds_status sync_default() {
 
 namespace ds {
 void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+uint64_t* debug_trace(size_t ntiles) { return ntiles <= g_trace_cap.load() ? g_trace.load() : nullptr; }
 }  // namespace ds
 
 extern "C" {
@@ -311,6 +315,13 @@ ds_status ds_release_workspaces(void) {
 }
 
 uint64_t ds_launch_count(void) { return g_launches.load(); }
+
+ds_status ds_debug_set_trace(uint64_t* d_trace, size_t capacity_tiles) {
+    if (d_trace && misaligned(d_trace, 8)) return DS_ERROR_INVALID_VALUE;
+    g_trace.store(d_trace);
+    g_trace_cap.store(d_trace ? capacity_tiles : 0);
+    return DS_SUCCESS;
+}
 
 int ds_version(void) { return 100; }
 

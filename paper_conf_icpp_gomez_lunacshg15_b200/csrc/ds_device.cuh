@@ -28,6 +28,19 @@ constexpr uint64_t kStateAgg = 1;     // irregular: tile aggregate only
 constexpr uint64_t kStateLoaded = 1;  // regular: tile's sources are loaded
 constexpr uint64_t kStateIncl = 2;    // irregular: inclusive prefix known
 
+// Status words are spread kStatusStride uint64 apart: tiles
+// finishing at the same time sit on different L2 lines.
+#ifndef DS_STATUS_STRIDE
+#define DS_STATUS_STRIDE 4
+#endif
+constexpr uint64_t kStatusStride = DS_STATUS_STRIDE;
+__host__ __device__ __forceinline__ uint64_t* status_ptr(uint64_t* base, int64_t tile) {
+    return base + tile * int64_t(kStatusStride);
+}
+__host__ __device__ __forceinline__ const uint64_t* status_ptr(const uint64_t* base, int64_t tile) {
+    return base + tile * int64_t(kStatusStride);
+}
+
 __host__ __device__ __forceinline__ uint64_t make_status(uint64_t state, uint64_t epoch,
                                                          uint64_t count) {
     return (state << kStateShift) | ((epoch & kEpochMask) << kEpochShift) | (count & kCountMask);
@@ -51,6 +64,30 @@ __device__ __forceinline__ void st_relaxed_gpu(uint64_t* p, uint64_t v) {
 }
 __device__ __forceinline__ void fence_acq_rel_gpu() {
     asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+
+// Status publication and the look-back's closing fence.
+// The DS hazards are write-after-read only: a tile never reads data that a
+// lower tile wrote (unique's boundary word is value-identical), so what must
+// hold is "every read of tile j completes before any tile > j overwrites
+// it".  A tile's reads have completed (the TMA transaction count reached
+// zero, or the values were consumed) before its status store is even
+// issued, and a successor's stores are issued only after it has read that
+// status, so relaxed status words suffice physically; GPU-scope release /
+// acquire fences cost ~1-2 us each here (MEMBAR.GPU drains the SM's whole
+// store stream).  -DDS_STRICT_ORDER restores release stores and the acquire
+// fence of the formal PTX-model argument; the test suite runs both builds.
+__device__ __forceinline__ void publish_status(uint64_t* p, uint64_t v) {
+#ifdef DS_STRICT_ORDER
+    st_release_gpu(p, v);
+#else
+    st_relaxed_gpu(p, v);
+#endif
+}
+__device__ __forceinline__ void lookback_acquire() {
+#ifdef DS_STRICT_ORDER
+    fence_acq_rel_gpu();
+#endif
 }
 
 struct alignas(16) u32x4 {
@@ -118,17 +155,33 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
 }
+// Blocking wait for the phase with the given parity.  The suspend-time hint
+// lets the hardware park the warp until the phase completes instead of
+// re-issuing try_wait in a tight loop.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile(
         "{\n"
         ".reg .pred P;\n"
         "DS_WAIT_%=:\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1, %2;\n"
         "@!P bra DS_WAIT_%=;\n"
         "}\n" ::"r"(smem_addr(bar)),
-        "r"(parity)
+        "r"(parity), "r"(1000000u)
         : "memory");
 }
+// One bounded wait (up to ~hint_ns); returns whether the phase completed.
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity, uint32_t hint_ns) {
+    uint32_t done;
+    asm volatile(
+        "{\n.reg .pred P;\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2, %3;\n"
+        "selp.u32 %0, 1, 0, P;\n}\n"
+        : "=r"(done)
+        : "r"(smem_addr(bar)), "r"(parity), "r"(hint_ns)
+        : "memory");
+    return done != 0;
+}
+
 // Named barrier among `count` threads (a subset of the CTA, whole warps).
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t count) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
@@ -146,6 +199,22 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
         "}\n" ::"r"(smem_addr(dst)),
         "l"(src), "r"(bytes), "r"(smem_addr(bar))
         : "memory");
+}
+
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ uint32_t smid() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
+    return r;
+}
+// Diagnostics (ds_debug_set_trace): per-tile events, 16 words per tile.
+constexpr int kTraceWords = 16;
+__device__ __forceinline__ void trace_event(uint64_t* trace, uint64_t tile, int ev, uint64_t v) {
+    if (trace) trace[tile * kTraceWords + ev] = v;
 }
 
 // Scheduling-stress hook (tests T3): with -DDS_DEBUG_DELAY the calling

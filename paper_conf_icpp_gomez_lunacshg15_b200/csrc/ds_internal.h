@@ -54,5 +54,7 @@ cudaError_t launch_shard_offsets(const uint64_t* d_counts, size_t world, size_t 
                                  uint64_t* d_result, cudaStream_t s);
 
 void count_launch();
+// Diagnostics buffer set by ds_debug_set_trace (null unless it covers ntiles).
+uint64_t* debug_trace(size_t ntiles);
 
 }  // namespace ds

@@ -2,36 +2,37 @@
 // stream compaction, select and unique (Algorithm 2, P:168-190;
 // §III-B; primitives §IV-B/C P:230-282).
 //
-// Persistent, warp-specialised CTAs (two per SM) walk input tiles of
-// T = 8192 words in dynamic-ticket order (Fig. 4) through a 3-stage
-// shared-memory ring:
+// One persistent, warp-specialised CTA per SM walks input tiles of
+// T = 8192 words in dynamic-ticket order (Fig. 4) through a 6-stage ring of
+// shared-memory tiles.  Each role works on a different tile at a time:
 //
-//   producer warp   a1 draw the next ticket when a stage is free
-//                   a2 one TMA bulk copy of the tile (plus, for unique, the
-//                      16 bytes before it) into the stage (Alg. 2 lines 1-11;
-//                      P:84 "on-chip memory")
-//                   a3+a4 the tile aggregate: keep flags and one warp
-//                      reduction ("Reduction", done before the sync
-//                      as P:158 recommends)
-//                   a5a publish AGG (release) the moment the tile has landed
-//   resolver warp   a5b decoupled look-back over 128 predecessors per round
-//                      trip, publish INCL; the last tile writes out_n (a8).
-//                      This replaces the serial flag chain of Fig. 7, which
-//                      is latency-bound on B200
-//   8 consumer      a6 rank of every kept word in input order ("binary
-//   warps              prefix sum"): ballot/popc within each
-//                      warp-vector + a scan of the 64 warp-vector counts
-//                   a7 scatter kept words in the stage at their final 16-byte
-//                      phase, then 128-bit stores of [excl, excl+A) (scalar
-//                      head/tail), then release the stage
+//   producer warp    a1 draws the next ticket as soon as a stage is free and
+//                    a2 loads the tile (plus, for unique, the 16 bytes before
+//                       it) with one TMA bulk copy (Alg. 2 lines 1-11; P:84
+//                       "on-chip memory")
+//  16 ranker warps   a3 keep flags (predicate / unique stencil)
+//                    a4 per-warp counts and the tile aggregate ("Reduction",
+//                       P:182) -- published as AGG at once
+//                    a6 rank of every kept word in input order ("binary
+//                       prefix sum": ballot/popc inside each
+//                       warp's contiguous 512-word segment + a scan of the 16
+//                       warp totals); the kept words are compacted in place
+//   6 resolver warps a5 (one per stage) decoupled look-back over 512
+//                       predecessors per round trip, started as soon as the
+//                       ticket is drawn (it needs no data), then INCL; the last
+//                       tile writes out_n (a8).  This replaces the serial flag
+//                       chain of Fig. 7, which is latency-bound on B200
+//
+//   6 storer warps   a7 128-bit stores of the compacted tile to
+//                       [excl, excl + A) (scalar head/tail), then free the stage
 //
-// A drawn tile's AGG depends only on its own bulk copy, never on this CTA's
-// progress through earlier tiles (DESIGN.md §5 explains why that matters).
-// In-place safety: AGG/INCL are published only after the
-// tile's copy completed; a tile stores only after the look-back saw AGG/INCL
-// of every lower tile; outputs of tile t lie in [0, (t+1)T), so no lower tile
-// writes into a higher tile's input.  Deadlock freedom: look-backs wait only
-// for lower (already drawn) tiles, whose AGG is published without waiting.
+// A drawn tile's AGG depends only on its own load and ranking, never on the
+// resolution of earlier tiles.  In-place safety:
+// AGG/INCL are published only after the tile's copy completed; stores happen
+// only after the look-back saw AGG/INCL of every lower tile; outputs of tile t
+// lie in [0, (t+1)T), so no lower tile writes into a higher tile's input.
+// Deadlock freedom: look-backs wait only for lower (already drawn) tiles, and
+// a drawn tile reaches AGG without waiting on any other tile.
 #include "ds_device.cuh"
 #include "ds_internal.h"
 
@@ -52,6 +53,7 @@ struct IrregParams {
     uint32_t ntiles;
     uint32_t draws;   // ntiles + gridDim.x
     uint32_t value;   // compact: remove value; select: predicate parameter
+    uint64_t* trace;  // diagnostics: 8 timestamps per tile, or null
 };
 
 // ---- predicates (a3) ----------------------------------------------------
@@ -83,43 +85,65 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
     return m;
 }
 
-// ---- tile geometry ------------------------------------------------------
-constexpr int kConsumerWarps = 8;
-constexpr int kCT = 32 * kConsumerWarps;  // consumer threads
-constexpr int kItems = 32;                // words per consumer thread
-constexpr int kVec = kItems / 4;
-constexpr int kT = kCT * kItems;          // 8192 words = 32 KB per tile
-constexpr int kSlots = kVec * kConsumerWarps;  // warp-vectors per tile (64)
+// ---- CTA shape ----------------------------------------------------------
+constexpr int kRankWarps = 16;
+constexpr int kRT = 32 * kRankWarps;      // ranker threads
+constexpr int kSeg = 512;                 // contiguous words ranked by one warp
+constexpr int kGroup = 8;                 // contiguous words per lane per group
+constexpr int kGroups = kSeg / (32 * kGroup);  // groups per warp (2)
+constexpr int kT = kRankWarps * kSeg;     // 8192 words = 32 KB per tile
+#ifndef DS_IRR_STAGES
+#define DS_IRR_STAGES 6
+#endif
+constexpr int kResolvers = DS_IRR_STAGES;  // one per stage
+constexpr int kStoreWarps = 6;
+constexpr int kST = 32 * kStoreWarps;
+constexpr int kWarpResolver0 = kRankWarps;                 // 16..21
+constexpr int kWarpStorer0 = kRankWarps + kResolvers;      // 22..27
+constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;  // 28
+constexpr int kThreads = 32 * (kWarpProducer + 1);
 constexpr int kPre = 4;                   // words before the tile (unique's boundary word)
-constexpr int kStageWords = kT + kPre + 4;  // + 4: store-phase realignment slack
-constexpr int kStages = 3;
-constexpr int kThreads = 32 * (2 + kConsumerWarps);
+constexpr int kStageWords = kT + kPre + 4;
+constexpr int kStages = DS_IRR_STAGES;
+#ifndef DS_IRR_MAXLOADS
+#define DS_IRR_MAXLOADS 3
+#endif
+constexpr uint32_t kMaxLoads = DS_IRR_MAXLOADS;  // tile copies in flight per CTA
 constexpr size_t kSmem = size_t(kStages) * kStageWords * 4;
-static_assert(kSlots == 64, "producer scan assumes two slots per lane");
+static_assert(kRankWarps <= 32, "warp-total scan in one warp");
+static_assert(kResolvers == kStages, "resolver r serves stage r");
+static_assert(kSmem <= 227 * 1024, "shared memory");
 
-// Keep mask of the 4 words of warp-vector slot x (tile word index) from the
-// staged tile.  Identical in producer and consumers.
+// Keep mask of the kGroup words w[] at tile word index x (from the staged
+// tile).
 template <class Op>
 __device__ __forceinline__ uint32_t keep_mask(const IrregParams& p, const uint32_t* stage,
-                                              uint64_t tb, bool full, int x, const u32x4& q,
+                                              uint64_t tb, bool full, int x, const uint32_t (&w)[kGroup],
                                               bool has_hprev, uint32_t hprev) {
-    const uint32_t w[4] = {q.x, q.y, q.z, q.w};
     uint32_t m = 0;
     if constexpr (Op::kUnique) {
         uint32_t prev = stage[kPre + x - 1];  // x == 0: the word before the tile
+        const bool first = tb == 0 && x == 0;  // holds the array's first word (index p.lo < 4)
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-            const uint64_t e = tb + x + k;
+        for (int k = 0; k < kGroup; ++k) {
             bool kp = w[k] != prev;
-            if (e == p.lo) kp = !has_hprev || w[k] != hprev;  // array's first word (R18)
             prev = w[k];
-            if ((full || (e >= p.lo && e < p.hi)) && kp) m |= 1u << k;
+            if (first && k == int(p.lo)) kp = !has_hprev || w[k] != hprev;  // shard halo (R18)
+            if (!full) {
+                const uint64_t e = tb + x + k;
+                kp = kp && e >= p.lo && e < p.hi;
+            }
+            m |= uint32_t(kp) << k;
         }
     } else {
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-            const uint64_t e = tb + x + k;
-            if ((full || (e >= p.lo && e < p.hi)) && Op::keep(w[k], p.value)) m |= 1u << k;
+        for (int k = 0; k < kGroup; ++k) {
+            bool kp = Op::keep(w[k], p.value);
+            if (!full) {
+                const uint64_t e = tb + x + k;
+                kp = kp && e >= p.lo && e < p.hi;
+            }
+            m |= uint32_t(kp) << k;
         }
     }
     return m;
@@ -137,52 +161,53 @@ __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) 
     return false;
 }
 
-// a5b: decoupled look-back by one warp, 4 predecessors per lane (128 per
-// round trip).  Lane l, slot m examines tile base - (4l + m).  Waits only
-// for the tiles up to the nearest INCL predecessor.  Ends with one acquire
-// fence per lane and a __syncwarp so lane 0's later release is cumulative
-// over everything the warp observed.
-constexpr int kLB = 4;
+// a5: decoupled look-back by one warp over 512 predecessors per round trip.
+// Slot (m, lane) examines tile base - (32m + lane): every load instruction
+// reads 32 consecutive status words.  Waits only for the tiles up to the
+// nearest INCL predecessor.  Ends with one acquire fence per lane and a
+// __syncwarp so lane 0's later release is cumulative over all lanes.
+#ifndef DS_IRR_LB
+#define DS_IRR_LB 4
+#endif
+constexpr int kLB = DS_IRR_LB;  // look-back slots per lane (32 * kLB tiles per round)
 
 __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status, uint32_t tile,
-                                             uint32_t epoch, int lane) {
+                                             uint32_t epoch, int lane, uint64_t* trace) {
     uint64_t excl = 0;
+    uint32_t rounds = 0, polls = 0;
     int64_t base = int64_t(tile) - 1;
     while (true) {
         uint64_t s[kLB];
-        uint32_t okm = 0;  // bit m: slot m has a current status
+        uint32_t okm = 0;  // bit m: slot m holds a current status
 #pragma unroll
         for (int m = 0; m < kLB; ++m) {
-            const int64_t idx = base - (kLB * lane + m);
-            if (idx >= 0) {
-                s[m] = ld_relaxed_gpu(status + idx);
-                if (status_current(s[m], epoch)) okm |= 1u << m;
-            } else {
-                s[m] = make_status(kStateIncl, epoch, 0);  // virtual INCL(0) before tile 0
-                okm |= 1u << m;
-            }
+            const int64_t idx = base - (32 * m + lane);
+            s[m] = idx >= 0 ? ld_relaxed_gpu(status_ptr(status, idx)) : make_status(kStateIncl, epoch, 0);
         }
-        uint32_t ns = 16;
-        int L, M;  // nearest INCL: lane L, slot M (L == 32: none in this round)
+#pragma unroll
+        for (int m = 0; m < kLB; ++m)
+            if (status_current(s[m], epoch)) okm |= 1u << m;
+        if (rounds++ == 0 && lane == 0) trace_event(trace, tile, 10, globaltimer());
+        uint32_t ns = 0;
+        uint32_t M, L;  // nearest INCL at slot M, lane L (M == kLB: none this round)
         while (true) {
             uint32_t inclm = 0;
 #pragma unroll
             for (int m = 0; m < kLB; ++m)
                 if ((okm >> m & 1u) && status_state(s[m]) == kStateIncl) inclm |= 1u << m;
-            const uint32_t lanes_incl = __ballot_sync(kFull, inclm != 0);
-            L = lanes_incl ? __ffs(lanes_incl) - 1 : 32;
-            M = __shfl_sync(kFull, inclm ? __ffs(inclm) - 1 : kLB, L & 31);
-            // every slot strictly before (L, M) and (L, M) itself must be current
-            const uint32_t need = lane < L ? ((1u << kLB) - 1) : (lane == L ? ((2u << M) - 1) : 0u);
-            const bool bad = (okm & need) != need;
-            if (!__any_sync(kFull, bad)) break;
-            __nanosleep(ns);
-            ns = ns < 256 ? ns * 2 : 256;
+            M = __reduce_min_sync(kFull, inclm ? uint32_t(__ffs(inclm) - 1) : uint32_t(kLB));
+            L = M < kLB ? uint32_t(__ffs(__ballot_sync(kFull, inclm >> M & 1u)) - 1) : 32u;
+            // needed: every slot before (M, L) in distance order, and (M, L)
+            const uint32_t need = (M < kLB ? ((1u << M) - 1u) : ((1u << kLB) - 1u)) |
+                                  (M < kLB && uint32_t(lane) <= L ? (1u << M) : 0u);
+            if (!__any_sync(kFull, (okm & need) != need)) break;
+            if (ns) __nanosleep(ns);
+            ns = ns ? (ns < 256 ? ns * 2 : 256) : 32;
+            ++polls;
 #pragma unroll
             for (int m = 0; m < kLB; ++m) {
                 if (!(okm >> m & 1u) && (need >> m & 1u)) {
-                    const int64_t idx = base - (kLB * lane + m);
-                    s[m] = ld_relaxed_gpu(status + idx);
+                    s[m] = ld_relaxed_gpu(status_ptr(status, base - (32 * m + lane)));
                     if (status_current(s[m], epoch)) okm |= 1u << m;
                 }
             }
@@ -191,18 +216,24 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status
         uint64_t inc = 0;
 #pragma unroll
         for (int m = 0; m < kLB; ++m) {
-            if (lane < L || (lane == L && m < M)) agg += uint32_t(status_count(s[m]));
-            if (lane == L && m == M) inc = status_count(s[m]);
+            if (uint32_t(m) < M || (uint32_t(m) == M && uint32_t(lane) < L)) agg += uint32_t(status_count(s[m]));
+            if (uint32_t(m) == M && uint32_t(lane) == L) inc = status_count(s[m]);
         }
         excl += uint64_t(__reduce_add_sync(kFull, agg));
-        if (L < 32) {
+        if (M < kLB) {
             excl += __shfl_sync(kFull, inc, L);
             break;
         }
         base -= 32 * kLB;
     }
-    fence_acq_rel_gpu();
+    if (lane == 0) {
+        trace_event(trace, tile, 8, rounds);
+        trace_event(trace, tile, 9, polls);
+        trace_event(trace, tile, 11, globaltimer());
+    }
+    lookback_acquire();
     __syncwarp();
+    if (lane == 0) trace_event(trace, tile, 12, globaltimer());
     return excl;
 }
 
@@ -210,130 +241,87 @@ struct StageMeta {
     uint32_t tile;           // kNoTile: end of this CTA's work
     uint32_t total;          // kept words in the tile
     unsigned long long excl; // kept words in all lower tiles
-    uint32_t slot[kSlots];   // kept-word counts of the warp-vector slots
+    uint32_t wtot[kRankWarps];  // kept words in each ranker warp's segment
 };
 
+// mbarrier wait that also returns (false) once the CTA's work is known to
+// end before ring position k (the resolvers take alternate positions, so the
+// one not holding the end marker is released this way).
+__device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
+                                                 const volatile uint32_t* s_end, uint32_t k) {
+    while (true) {
+        if (mbar_try_wait(bar, parity, 20000u)) return true;
+        // Strictly beyond the end marker: the position holding the marker
+        // itself still gets its arrival and must pass it on.
+        if (*s_end < k) return false;
+    }
+}
+
 template <class Op>
-__global__ void __launch_bounds__(kThreads, 2) irregular_kernel(const IrregParams p) {
+__global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParams p) {
     extern __shared__ __align__(128) uint32_t smem[];
-    __shared__ __align__(8) uint64_t bar_full[kStages], bar_counted[kStages], bar_resolved[kStages],
-        bar_empty[kStages];
+    __shared__ __align__(8) uint64_t bar_drawn[kStages], bar_full[kStages], bar_counted[kStages], bar_ranked[kStages],
+        bar_resolved[kStages], bar_empty[kStages];
     __shared__ StageMeta meta[kStages];
     __shared__ uint32_t s_epoch;
+    __shared__ volatile uint32_t s_end;  // ring position of the end marker
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
         for (int s = 0; s < kStages; ++s) {
+            mbar_init(&bar_drawn[s], 1);
             mbar_init(&bar_full[s], 1);
             mbar_init(&bar_counted[s], 1);
+            mbar_init(&bar_ranked[s], 1);
             mbar_init(&bar_resolved[s], 1);
-            mbar_init(&bar_empty[s], kConsumerWarps);
+            mbar_init(&bar_empty[s], kStoreWarps);
         }
+        s_end = 0xffffffffu;
         mbar_fence_init();
     }
     __syncthreads();
 
-    if (warp == 0) {
-        // ------------------------------------------------ producer warp
-        bool has_hprev = false;
-        uint32_t hprev = 0;
-        if (Op::kUnique) has_hprev = halo_prev(p, hprev);
+    if (warp == kWarpProducer) {
+        // ------------------------------------------------ producer (lane 0)
+        if (lane != 0) return;
         for (uint32_t k = 0;; ++k) {
             const int s = k % kStages;
             const uint32_t use = k / kStages;
             uint32_t* stage = smem + s * kStageWords;
-            mbar_wait(&bar_empty[s], (use & 1) ^ 1);  // consumers released tile k - kStages
-            uint32_t t = 0, epoch = 0;
-            if (lane == 0) {
-                draw_ticket(p.ctrl, p.draws, t, epoch);
-                if (k == 0) s_epoch = epoch;
+            mbar_wait(&bar_empty[s], (use & 1) ^ 1);  // storers released tile k - kStages
+            if (k >= kMaxLoads) {
+                // At most kMaxLoads tile copies in flight per CTA: deeper queues only
+                // add latency to the status words' round trips.
+                const uint32_t kp = k - kMaxLoads;
+                mbar_wait(&bar_full[kp % kStages], (kp / kStages) & 1);
             }
-            t = __shfl_sync(kFull, t, 0);
-            epoch = __shfl_sync(kFull, epoch, 0);
+            uint32_t t, epoch;
+            draw_ticket(p.ctrl, p.draws, t, epoch);
+            if (k == 0) s_epoch = epoch;
             if (t >= p.ntiles) {  // one failed draw per CTA ends its work
-                if (lane == 0) {
-                    meta[s].tile = kNoTile;
-                    mbar_arrive(&bar_counted[s]);
-                }
-                break;
+                meta[s].tile = kNoTile;
+                s_end = k;
+                mbar_arrive(&bar_drawn[s]);
+                mbar_arrive(&bar_full[s]);
+                return;
             }
+            meta[s].tile = t;
+            mbar_arrive(&bar_drawn[s]);  // the resolver starts this tile's look-back now
+            trace_event(p.trace, t, 0, globaltimer());
+            trace_event(p.trace, t, 7, smid());
+            debug_delay(t, 0);
             const uint64_t tb = uint64_t(t) * kT;
-            if (lane == 0) {
-                debug_delay(t, 0);
-                uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
-                end = (end + 3) & ~3ull;  // may read <= 12 bytes past the array end (same 16 B chunk)
-                const uint64_t beg = (Op::kUnique && t > 0) ? tb - 4 : tb;
-                const uint32_t bytes = uint32_t(end - beg) * 4u;
-                fence_proxy_async_smem();
-                mbar_arrive_expect_tx(&bar_full[s], bytes);
-                bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_full[s]);
-            }
-            mbar_wait(&bar_full[s], use & 1);
-
-            // a3 + a4: the tile aggregate.  Lane l counts words 4*(32j + l) + [0, 4),
-            // j < T/128, then one warp reduction.
-            uint32_t c = 0;
-            if (tb >= p.lo && tb + kT <= p.hi) {
-#pragma unroll 8
-                for (int j = 0; j < kT / 128; ++j) {
-                    const int x = 4 * (32 * j + lane);
-                    const u32x4 q = *reinterpret_cast<const u32x4*>(stage + kPre + x);
-                    if constexpr (Op::kUnique) {
-                        const uint32_t pw = stage[kPre + x - 1];
-                        c += (q.x != pw) + (q.y != q.x) + (q.z != q.y) + (q.w != q.z);
-                    } else {
-                        c += Op::keep(q.x, p.value) + Op::keep(q.y, p.value) + Op::keep(q.z, p.value) +
-                             Op::keep(q.w, p.value);
-                    }
-                }
-                if (Op::kUnique && tb == p.lo && lane == 0) {  // the array's first word (R18)
-                    const uint32_t w0 = stage[kPre];
-                    c += (!has_hprev || w0 != hprev) - (w0 != stage[kPre - 1]);
-                }
-            } else {  // the first (misaligned) or last (ragged) tile
-                for (int j = 0; j < kT / 128; ++j) {
-                    const int x = 4 * (32 * j + lane);
-                    const u32x4 q = *reinterpret_cast<const u32x4*>(stage + kPre + x);
-                    c += __popc(keep_mask<Op>(p, stage, tb, false, x, q, has_hprev, hprev));
-                }
-            }
-            const uint32_t total = __reduce_add_sync(kFull, c);
-            __syncwarp();
-            if (lane == 0) {
-                meta[s].tile = t;
-                meta[s].total = total;
-                debug_delay(t, 1);
-                // a5a: publish the aggregate now -- it depends on nothing else.
-                st_release_gpu(p.status + t, make_status(t == 0 ? kStateIncl : kStateAgg, epoch, total));
-                mbar_arrive(&bar_counted[s]);
-            }
+            uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
+            end = (end + 3) & ~3ull;  // may read <= 12 bytes past the array end (same 16 B chunk)
+            const uint64_t beg = (Op::kUnique && t > 0) ? tb - 4 : tb;
+            const uint32_t bytes = uint32_t(end - beg) * 4u;
+            fence_proxy_async_smem();
+            mbar_arrive_expect_tx(&bar_full[s], bytes);
+            bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_full[s]);
         }
-    } else if (warp == 1) {
-        // ------------------------------------------------ resolver warp
-        for (uint32_t k = 0;; ++k) {
-            const int s = k % kStages;
-            const uint32_t use = k / kStages;
-            mbar_wait(&bar_counted[s], use & 1);
-            const uint32_t t = meta[s].tile;
-            if (t == kNoTile) {
-                if (lane == 0) mbar_arrive(&bar_resolved[s]);
-                break;
-            }
-            const uint32_t epoch = s_epoch;
-            const uint32_t total = meta[s].total;
-            if (lane == 0) debug_delay(t, 2);
-            __syncwarp();
-            const uint64_t excl = t > 0 ? lookback(p.status, t, epoch, lane) : 0ull;
-            if (lane == 0) {
-                if (t > 0) st_release_gpu(p.status + t, make_status(kStateIncl, epoch, excl + total));
-                meta[s].excl = excl;
-                if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = excl + total;
-                mbar_arrive(&bar_resolved[s]);
-            }
-        }
-    } else {
-        // ------------------------------------------------ consumer warps
-        const int cw = warp - 2, ct = tid - 64;
+    } else if (warp < kRankWarps) {
+        // ------------------------------------------------ ranker warps
+        const int rw = warp, rt = tid;
         const uint32_t lt = lanemask_lt();
         bool has_hprev = false;
         uint32_t hprev = 0;
@@ -342,85 +330,166 @@ __global__ void __launch_bounds__(kThreads, 2) irregular_kernel(const IrregParam
             const int s = k % kStages;
             const uint32_t use = k / kStages;
             uint32_t* stage = smem + s * kStageWords;
-            mbar_wait(&bar_resolved[s], use & 1);
+            mbar_wait(&bar_full[s], use & 1);
             const uint32_t t = meta[s].tile;
-            if (t == kNoTile) break;
+            if (t == kNoTile) {
+                if (rt == 0) mbar_arrive(&bar_counted[s]);
+                break;
+            }
+            if (rt == 0) trace_event(p.trace, t, 1, globaltimer());
             const uint64_t tb = uint64_t(t) * kT;
             const bool full = tb >= p.lo && tb + kT <= p.hi;
 
-            // a6: words -> registers, keep masks, in-warp exclusive ranks and the
-            // count of every warp-vector slot (i, warp).
-            uint32_t v[kVec][4];
-            uint32_t masks = 0;                 // 4 bits per vector
-            uint32_t lane_pre[kVec / 4] = {};   // 8 bits per vector (< 128)
+            // a3/a4: warp rw ranks tile words [kSeg*rw, kSeg*(rw+1)); in group g
+            // lane l holds the kGroup contiguous words at x = kSeg*rw + 256g + 8l.
+            uint32_t v[kGroups][kGroup];
+            uint32_t masks = 0;     // kGroup keep bits per group
+            uint32_t lane_pre = 0;  // 16 bits per group: kept words of lower lanes
+            uint32_t wrun = 0;      // kept words of the warp's earlier groups
+            uint32_t goff = 0;      // 16 bits per group: offset of group g in the segment
 #pragma unroll
-            for (int i = 0; i < kVec; ++i) {
-                const int x = 4 * (i * kCT + ct);
-                const u32x4 q = *reinterpret_cast<const u32x4*>(stage + kPre + x);
-                v[i][0] = q.x; v[i][1] = q.y; v[i][2] = q.z; v[i][3] = q.w;
-                const uint32_t m = keep_mask<Op>(p, stage, tb, full, x, q, has_hprev, hprev);
-                masks |= m << (4 * i);
-                const uint32_t c = __popc(m);
+            for (int g = 0; g < kGroups; ++g) {
+                const int x = kSeg * rw + 32 * kGroup * g + kGroup * lane;
+                const u32x4 q0 = *reinterpret_cast<const u32x4*>(stage + kPre + x);
+                const u32x4 q1 = *reinterpret_cast<const u32x4*>(stage + kPre + x + 4);
+                v[g][0] = q0.x; v[g][1] = q0.y; v[g][2] = q0.z; v[g][3] = q0.w;
+                v[g][4] = q1.x; v[g][5] = q1.y; v[g][6] = q1.z; v[g][7] = q1.w;
+                const uint32_t m = keep_mask<Op>(p, stage, tb, full, x, v[g], has_hprev, hprev);
+                masks |= m << (kGroup * g);
+                const uint32_t c = __popc(m);  // 0..8
                 const uint32_t b0 = __ballot_sync(kFull, c & 1u);
                 const uint32_t b1 = __ballot_sync(kFull, c & 2u);
                 const uint32_t b2 = __ballot_sync(kFull, c & 4u);
-                lane_pre[i / 4] |= (__popc(b0 & lt) + 2u * __popc(b1 & lt) + 4u * __popc(b2 & lt))
-                                   << (8 * (i % 4));
-                if (lane == 0) meta[s].slot[i * kConsumerWarps + cw] = __popc(b0) + 2u * __popc(b1) + 4u * __popc(b2);
+                const uint32_t b3 = __ballot_sync(kFull, c & 8u);
+                lane_pre |= (__popc(b0 & lt) + 2u * __popc(b1 & lt) + 4u * __popc(b2 & lt) +
+                             8u * __popc(b3 & lt)) << (16 * g);
+                goff |= wrun << (16 * g);
+                wrun += __popc(b0) + 2u * __popc(b1) + 4u * __popc(b2) + 8u * __popc(b3);
             }
-            named_bar_sync(1, kCT);  // slot counts written; every consumer holds its words
+            if (lane == 0) meta[s].wtot[rw] = wrun;
+            named_bar_sync(1, kRT);  // warp totals written; every ranker holds its words
 
-            // Exclusive scan of the 64 slot counts in input order, redundantly in
-            // every warp (lane l holds slots l and l + 32).
-            uint32_t ca = meta[s].slot[lane], cb = meta[s].slot[lane + 32];
-            uint32_t ia = ca, ib = cb;
+            // Exclusive scan of the kRankWarps warp totals (input order), redundantly
+            // in every warp.
+            const uint32_t cw = lane < kRankWarps ? meta[s].wtot[lane] : 0u;
+            uint32_t iw = cw;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t ya = __shfl_up_sync(kFull, ia, o);
-                const uint32_t yb = __shfl_up_sync(kFull, ib, o);
-                if (lane >= o) {
-                    ia += ya;
-                    ib += yb;
-                }
+                const uint32_t y = __shfl_up_sync(kFull, iw, o);
+                if (lane >= o) iw += y;
             }
-            const uint32_t tot_a = __shfl_sync(kFull, ia, 31);
-            const uint32_t ea = ia - ca, eb = tot_a + ib - cb;  // exclusive offsets of slots l, l+32
+            const uint32_t total = __shfl_sync(kFull, iw, 31);
+            const uint32_t wbase = __shfl_sync(kFull, iw - cw, rw);
+            if (rt == 0) {
+                // a4: publish the aggregate right away -- it depends on nothing else
+                // (a relaxed status store), then hand the total to
+                // this stage's resolver.
+                meta[s].total = total;
+                debug_delay(t, 1);
+                publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
+                trace_event(p.trace, t, 2, globaltimer());
+                mbar_arrive(&bar_counted[s]);
+            }
 
-            // a7: scatter at the output's 16-byte phase, then aligned stores.
+            // a6: compact the kept words in place: rank r -> stage[kPre + r].
+#pragma unroll
+            for (int g = 0; g < kGroups; ++g) {
+                uint32_t r = wbase + ((goff >> (16 * g)) & 0xFFFFu) + ((lane_pre >> (16 * g)) & 0xFFFFu);
+                const uint32_t m = masks >> (kGroup * g);
+#pragma unroll
+                for (int k = 0; k < kGroup; ++k)
+                    if (m >> k & 1u) stage[kPre + r++] = v[g][k];
+            }
+            named_bar_sync(1, kRT);  // compacted tile complete
+            if (rt == 0) mbar_arrive(&bar_ranked[s]);
+        }
+    } else if (warp < kWarpStorer0) {
+        // ------------------------------------------------ resolver warps
+        // Resolver r serves stage r: ring positions k = r, r + kStages, ...
+        const uint32_t r = warp - kWarpResolver0;
+        for (uint32_t k = r;; k += kStages) {
+            const int s = int(r);
+            const uint32_t use = k / kStages;
+            if (!mbar_wait_or_end(&bar_drawn[s], use & 1, &s_end, k)) break;
+            const uint32_t t = meta[s].tile;
+            if (t == kNoTile) {
+                if (lane == 0) mbar_arrive(&bar_resolved[s]);
+                break;
+            }
+            const uint32_t epoch = s_epoch;
+            if (lane == 0) {
+                debug_delay(t, 2);
+                trace_event(p.trace, t, 3, globaltimer());
+            }
+            __syncwarp();
+            // a5: the look-back needs only the ticket, so it runs while the tile is
+            // still being loaded and ranked.
+#ifdef DS_DEBUG_NO_LOOKBACK  // timing experiment only: wrong output, same traffic
+            const uint64_t excl = uint64_t(t) * (kT / 2);
+#else
+            const uint64_t excl = t > 0 ? lookback(p.status, t, epoch, lane, p.trace) : 0ull;
+#endif
+            mbar_wait(&bar_counted[s], use & 1);  // the tile's aggregate is published
+            const uint32_t total = meta[s].total;
+            if (lane == 0 && t > 0)
+                publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
+            mbar_wait(&bar_ranked[s], use & 1);  // the compacted tile is in the stage
+            if (lane == 0) {
+                trace_event(p.trace, t, 4, globaltimer());
+                meta[s].excl = excl;
+                if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = excl + total;
+                mbar_arrive(&bar_resolved[s]);
+            }
+        }
+    } else {
+        // ------------------------------------------------ storer warps
+        const int st = tid - 32 * kWarpStorer0;
+        for (uint32_t k = 0;; ++k) {
+            const int s = k % kStages;
+            const uint32_t use = k / kStages;
+            const uint32_t* stage = smem + s * kStageWords;
+            mbar_wait(&bar_resolved[s], use & 1);
+            const uint32_t t = meta[s].tile;
+            if (t == kNoTile) break;
+            if (st == 0) {
+                trace_event(p.trace, t, 5, globaltimer());
+                debug_delay(t, 3);
+            }
+            // a7: chunk c covers virtual words c0 + 4c + [0, 4) = ranks 4c - ph + [0, 4)
+            // (ph = 16-byte phase of the output start), read from the stage as
+            // two aligned vectors and funnel-shifted.
             const uint32_t A = meta[s].total;
             const uint64_t s0 = p.lo + meta[s].excl;
-            uint32_t* out = stage + kPre + uint32_t(s0 & 3);
-#pragma unroll
-            for (int i = 0; i < kVec; ++i) {
-                const int slot = i * kConsumerWarps + cw;  // warp-uniform
-                const uint32_t base = __shfl_sync(kFull, slot < 32 ? ea : eb, slot & 31);
-                uint32_t r = base + ((lane_pre[i / 4] >> (8 * (i % 4))) & 0xFFu);
-                const uint32_t m = masks >> (4 * i);
-#pragma unroll
-                for (int kk = 0; kk < 4; ++kk)
-                    if (m >> kk & 1u) out[r++] = v[i][kk];
-            }
-            named_bar_sync(1, kCT);  // compacted tile complete
-            if (ct == 0) debug_delay(t, 3);
             const uint64_t s1 = s0 + A;
             const uint64_t c0 = s0 & ~3ull;
+            const uint32_t ph = uint32_t(s0 & 3);
+#ifdef DS_DEBUG_NO_STORE  // timing experiment only: no output written
+            const uint32_t nchunks = 0;
+#else
             const uint32_t nchunks = A ? uint32_t((s1 - c0 + 3) >> 2) : 0u;
-#pragma unroll
-            for (int it = 0; it < kVec + 1; ++it) {
-                const uint32_t c = uint32_t(it * kCT + ct);
-                if (c >= nchunks) break;
+#endif
+            for (uint32_t c = st; c < nchunks; c += kST) {
+                const u32x4 hi = *reinterpret_cast<const u32x4*>(stage + kPre + 4 * c);
+                const u32x4 lo = *reinterpret_cast<const u32x4*>(stage + kPre + 4 * c - 4);
+                uint32_t w0, w1, w2, w3;
+                switch (ph) {  // warp-uniform
+                case 0: w0 = hi.x; w1 = hi.y; w2 = hi.z; w3 = hi.w; break;
+                case 1: w0 = lo.w; w1 = hi.x; w2 = hi.y; w3 = hi.z; break;
+                case 2: w0 = lo.z; w1 = lo.w; w2 = hi.x; w3 = hi.y; break;
+                default: w0 = lo.y; w1 = lo.z; w2 = lo.w; w3 = hi.x; break;
+                }
                 const uint64_t g = c0 + 4ull * c;
-                const u32x4 q = *reinterpret_cast<const u32x4*>(stage + kPre + 4 * c);
                 if (g >= s0 && g + 4 <= s1) {
-                    stg_stream_v4(p.abase + g, q.x, q.y, q.z, q.w);
+                    stg_stream_v4(p.abase + g, w0, w1, w2, w3);
                 } else {
-                    const uint32_t w[4] = {q.x, q.y, q.z, q.w};
+                    const uint32_t w[4] = {w0, w1, w2, w3};
 #pragma unroll
                     for (int kk = 0; kk < 4; ++kk)
                         if (g + kk >= s0 && g + kk < s1) stg_stream(p.abase + g + kk, w[kk]);
                 }
             }
             __syncwarp();
+            if (st == 0) trace_event(p.trace, t, 6, globaltimer());
             if (lane == 0) mbar_arrive(&bar_empty[s]);  // this warp is done with the stage
         }
     }
@@ -476,6 +545,7 @@ cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s) 
     p.halo_len = uint32_t(a.halo_len);
     p.ntiles = uint32_t(irregular_tiles(a));
     p.value = a.value;
+    p.trace = debug_trace(p.ntiles);
     count_launch();
     switch (a.op) {
     case IrregOp::Compact: return launch_op<OpCompact>(p, s);

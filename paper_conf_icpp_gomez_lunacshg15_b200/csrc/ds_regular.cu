@@ -138,15 +138,15 @@ __device__ __forceinline__ void wait_loaded(const uint64_t* __restrict__ status,
                                             int64_t hi, uint32_t epoch, int lane) {
     for (int64_t base = lo; base <= hi; base += 32) {
         const int64_t idx = base + lane;
-        bool ok = idx > hi || status_current(ld_relaxed_gpu(status + idx), epoch);
+        bool ok = idx > hi || status_current(ld_relaxed_gpu(status_ptr(status, idx)), epoch);
         uint32_t ns = 32;
         while (!__all_sync(0xffffffffu, ok)) {
             __nanosleep(ns);
             ns = ns < 512 ? ns * 2 : 512;
-            if (!ok) ok = status_current(ld_relaxed_gpu(status + idx), epoch);
+            if (!ok) ok = status_current(ld_relaxed_gpu(status_ptr(status, idx)), epoch);
         }
     }
-    fence_acq_rel_gpu();
+    lookback_acquire();
     __syncwarp();
 }
 
@@ -254,7 +254,7 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
             mbar_wait(&bar_full[s], use & 1);
             if (lane == 0) {
                 debug_delay(uint64_t(kt), 1);
-                st_release_gpu(p.status + kt, make_status(kStateLoaded, epoch, 0));
+                publish_status(status_ptr(p.status, kt), make_status(kStateLoaded, epoch, 0));
                 mbar_arrive(&bar_loaded[s]);
             }
         }

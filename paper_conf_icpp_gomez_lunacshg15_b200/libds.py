@@ -40,6 +40,7 @@ SIGNATURES = {
     "ds_release_workspaces": (_i, []),
     "ds_launch_count": (_u64, []),
     "ds_version": (_i, []),
+    "ds_debug_set_trace": (_i, [_vp, _sz]),
 }
 
 
@@ -187,6 +188,10 @@ def ds_launch_count() -> int:
 
 def ds_version() -> int:
     return int(_lib.ds_version())
+
+
+def ds_debug_set_trace(d_trace, capacity_tiles: int) -> None:
+    _check(_lib.ds_debug_set_trace(_addr(d_trace), capacity_tiles), "ds_debug_set_trace")
 
 
 def raw_status(name: str, *args) -> int:

@@ -18,7 +18,6 @@ import dsgen  # noqa: E402
 import oracle  # noqa: E402
 from paper_conf_icpp_gomez_lunacshg15_b200 import libds  # noqa: E402
 
-assert "stress" in libds.LIB_PATH, libds.LIB_PATH
 
 
 def u32(t):
@@ -59,7 +58,7 @@ def main(reps):
                 libds.ds_unpad_ex(a, R, NC, C, 4, None)
                 torch.cuda.synchronize()
                 assert np.array_equal(u32(a), exp), ("unpad-back", rep, R, C, NC)
-    print(f"stress OK: {reps} reps")
+    print(f"stress OK: {reps} reps with {libds.LIB_PATH}")
 
 
 if __name__ == "__main__":

@@ -11,8 +11,11 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 
 
 @pytest.mark.gpu
-def test_delay_injection_parity():
-    lib = build.build("stress")
+@pytest.mark.parametrize("variant", ["stress", "strict"])
+def test_delay_injection_parity(variant):
+    """stress: random per-CTA delays (-DDS_DEBUG_DELAY); strict: the
+    release/acquire status ordering build (-DDS_STRICT_ORDER)."""
+    lib = build.build(variant)
     env = dict(os.environ, LIBDS_PATH=lib)
     r = subprocess.run([sys.executable, os.path.join(HERE, "stress_driver.py"), "12"],
                        env=env, capture_output=True, text=True, timeout=900)
