@@ -1,0 +1,429 @@
+"""bench.py -- libds on B200: effective HBM GB/s of the in-place Data Sliding path.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl libds|reference]
+                    [--no-rows] [--no-e2e] [--no-cpu]
+    python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 \\
+        --master-port P bench.py --gpus N ...
+
+Headline (BASELINE.json configs[4], C5): sharded in-place stream compaction of
+4G int32 words (2^32, 16 GiB), 50 % kept, contiguous shards over N GPUs
+(strong scaling).  One step = on every rank: ds_compact_ex on its shard (the
+irregular DS kernel), NCCL all-gather of the 8-byte
+counts, ds_shard_offsets (global offset + out_n).  Between steps, outside the
+timed events, the pristine shard is restored (D2D copy) and L2 is flushed by
+reading a 512 MiB buffer.  value = sum over ranks of 4*(n_r + out_r) bytes /
+max-over-ranks device time of the step.
+
+rows (N == 1 only): the other BASELINE configs through the same C ABI --
+C1 compact 1M, C2 pad / unpad 4000x3990 <-> 4000, C3 select and unique on
+256M over f = 0..1, C4 compact 1G float32 at 10/50/90 %.
+
+--impl reference: the CPU oracle (oracle/, sequential C, one core) on a
+bounded sample of the same workload, rank 0 only.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "effective GB/s (read+write) and % of HBM peak for in-place compact/pad, 1/2/4/8 B200"
+N_TOTAL = 1 << 32
+FRAC = 0.5
+SEED = 0xD5201500 + 16 * 4  # dsgen.seed_for(4): C5
+WORKLOAD = "C5: sharded in-place stream compaction of 4G int32 (2^32 words), 50% kept, remove_value 0"
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
+            pk = json.load(fh)
+        return float(pk["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy_)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_ncu_traffic():
+    """DRAM bytes per launch of the headline kernel from the committed ncu capture."""
+    path = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(path) as fh:
+            d = json.load(fh)
+        return d.get("headline", {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.proc = None
+        self.gpu = gpu_index
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.12)
+        self.proc.terminate()
+        out, _ = self.proc.communicate(timeout=10)
+        sm, smax, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": smax,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def timed(fn, stream, restore=None, flush=None, reps=5, warmup=2):
+    """Median device time (ms) of fn() on `stream`, events around fn only."""
+    import torch
+    ts = []
+    for r in range(warmup + reps):
+        if restore:
+            restore()
+        if flush:
+            flush()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        fn()
+        b.record(stream)
+        b.synchronize()
+        if r >= warmup:
+            ts.append(a.elapsed_time(b))
+    return statistics.median(ts)
+
+
+def bench_rows(peak, flush):
+    """The other BASELINE configs (rank 0, N == 1)."""
+    import torch
+
+    import dsgen
+    from paper_conf_icpp_gomez_lunacshg15_b200 import libds
+    s = torch.cuda.current_stream()
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    rows = []
+
+    def row(op, cfg, ms, nbytes, extra=None):
+        gbs = nbytes / (ms * 1e-3) / 1e9
+        r = {"op": op, "config": cfg, "us": round(ms * 1e3, 2), "gbs": round(gbs, 1),
+             "frac": round(gbs / peak, 4)}
+        if extra:
+            r.update(extra)
+        rows.append(r)
+
+    def irregular(op, name, src, call, reps=5):
+        work = torch.empty_like(src)
+        ms = timed(lambda: call(work), s, restore=lambda: work.copy_(src), flush=flush, reps=reps)
+        m = int(d_n.item())
+        row(op, name, ms, 4 * (src.numel() + m), {"n": src.numel(), "out_n": m})
+
+    # C1: 1M int32 compaction, 50 %
+    n = 1 << 20
+    src = dsgen.compact_input(n, 0.5, dsgen.seed_for(0), device="cuda")
+    irregular("compact", "C1 1M int32 f=0.5", src,
+              lambda w: libds.ds_compact_ex(w, n, 0, d_n, None), reps=20)
+    # C2: pad 4000x3990 -> 4000 f32 and unpad back
+    R, C, NC = 4000, 3990, 4000
+    src = dsgen.matrix_input(R, C, NC, 4, kind="f32", device="cuda")
+    work = torch.empty_like(src)
+    ms = timed(lambda: libds.ds_pad_ex(work, R, C, NC, 4, None, None), s,
+               restore=lambda: work.copy_(src), flush=flush, reps=20)
+    row("pad", "C2 4000x3990->4000 f32", ms, 4 * (R * C + R * NC))
+    padded = src.clone()
+    libds.ds_pad(padded, R, C, NC, 4)
+    ms = timed(lambda: libds.ds_unpad_ex(work, R, NC, C, 4, None), s,
+               restore=lambda: work.copy_(padded), flush=flush, reps=20)
+    row("unpad", "C2 4000x4000->3990 f32", ms, 4 * (2 * R * C))
+    # C3: select (x > t) and unique, 256M int32, f = 0 .. 1
+    n = 1 << 28
+    src = dsgen.select_input(n, dsgen.seed_for(2), device="cuda")
+    for i in range(11):
+        f = i / 10
+        t = dsgen.select_threshold(f) & 0xFFFFFFFF
+        irregular("select", f"C3 256M int32 x>t f={f:.1f}", src,
+                  lambda w, t=t: libds.ds_select_ex(w, n, libds.DS_PRED_I32_GT, t, d_n, None), reps=3)
+    del src
+    for i in range(11):
+        f = i / 10
+        src = dsgen.unique_runs_input(n, f, dsgen.seed_for(2, 11 + i), device="cuda")
+        irregular("unique", f"C3 256M int32 runs f={f:.1f}", src,
+                  lambda w: libds.ds_unique_ex(w, n, None, 0, d_n, None), reps=3)
+        del src
+    # C4: 1G float32 compaction at 10 / 50 / 90 %
+    n = 1 << 30
+    for f in (0.1, 0.5, 0.9):
+        src = dsgen.compact_input(n, f, dsgen.seed_for(3, int(f * 10)), kind="f32", device="cuda")
+        irregular("compact", f"C4 1G f32 f={f}", src,
+                  lambda w: libds.ds_compact_ex(w, n, 0, d_n, None), reps=3)
+        del src
+    return rows
+
+
+def oracle_sample_input(n_sample):
+    import numpy as np
+
+    import dsgen
+    return dsgen.compact_input(n_sample, FRAC, SEED).numpy().view(np.uint32)
+
+
+def cpu_oracle_sample(n_sample, reps, src=None):
+    """The oracle (sequential C, 1 core) on a prefix-shaped sample of C5."""
+    import oracle
+    if src is None:
+        src = oracle_sample_input(n_sample)
+    ts, m = [], 0
+    for _ in range(reps):
+        a = src.copy()
+        t0 = time.perf_counter()
+        m = oracle.compact(a, 0)
+        ts.append(time.perf_counter() - t0)
+    t = statistics.median(ts)
+    gbs = 4 * (n_sample + m) / t / 1e9
+    return gbs, t, m
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    n_sample = 1 << 26
+    src = oracle_sample_input(n_sample)
+    steps = []
+    for i in range(args.warmup + args.steps):
+        gbs, t, m = cpu_oracle_sample(n_sample, 1, src)
+        if i >= args.warmup:
+            steps.append((gbs, t))
+    value = statistics.median(g for g, _ in steps)
+    ms = statistics.median(t for _, t in steps) * 1e3
+    sample = (f"one step = oracle_compact on a 2^26-word (256 MiB) sample of the C5 recipe "
+              f"(seed {SEED:#x}, f={FRAC}); 1 thread")
+    line = {"metric": METRIC, "value": round(value, 3), "unit": "GB/s", "impl": "reference",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic (counter-based hash, dsgen)",
+            "config": {"workload": WORKLOAD, "sample_words": n_sample},
+            "cpu_baseline": {"value": round(value, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": round(value, 3), "unit": "GB/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_libds(args):
+    import torch
+    import torch.distributed as dist
+
+    import dsgen
+    from paper_conf_icpp_gomez_lunacshg15_b200 import libds
+    from paper_conf_icpp_gomez_lunacshg15_b200.dist import ShardedDS, shard_range
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    peak, peak_src = load_peaks()
+
+    # ---- the rank's shard of the C5 array (generated in place, seeded by global index)
+    lo, hi = shard_range(N_TOTAL, world, rank)
+    n = hi - lo
+    pristine = torch.empty(n, dtype=torch.int32, device=dev)
+    for s0 in range(0, n, 1 << 27):
+        c = min(1 << 27, n - s0)
+        h = dsgen.hash_range(SEED, lo + s0, c, device=dev)
+        keep = dsgen._hi32(h) < dsgen.keep_threshold(FRAC)
+        val = dsgen._as_i32(dsgen._lo32(h) | 1)
+        pristine[s0:s0 + c] = torch.where(keep, val, torch.zeros_like(val))
+        del h, keep, val
+    work = torch.empty_like(pristine)
+    flush_buf = torch.empty(1 << 27, dtype=torch.int32, device=dev)  # 512 MiB > 126 MB L2
+    flush = lambda: flush_buf.sum()  # noqa: E731  (read-only flush: leaves no dirty lines)
+    stream = torch.cuda.current_stream()
+    ds = ShardedDS(device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def step_once(kernel_ev):
+        a, b, c = kernel_ev
+        a.record(stream)
+        libds.ds_compact_ex(work, n, 0, ds.d_count, stream)
+        b.record(stream)
+        ds._finish(stream)
+        c.record(stream)
+
+    def one_step(timed_events):
+        work.copy_(pristine)
+        flush()
+        step_once(timed_events)
+
+    # ---- warm-up
+    for _ in range(args.warmup):
+        one_step([torch.cuda.Event(enable_timing=True) for _ in range(3)])
+    barrier()
+
+    # ---- timed region: exactly K steps, barrier + sync on both sides
+    clocks = ClockSampler(local)
+    clocks.start()
+    launches0 = libds.ds_launch_count()
+    evs = []
+    barrier()
+    for _ in range(args.steps):
+        e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+        one_step(e)
+        evs.append(e)
+    barrier()
+    launches = libds.ds_launch_count() - launches0
+    clk = clocks.stop()
+    step_ms = sum(e[0].elapsed_time(e[2]) for e in evs)
+    kern_ms = sum(e[0].elapsed_time(e[1]) for e in evs) / args.steps
+    out_n = int(ds.d_count.item())
+    total_out = int(ds.d_result[1].item())
+    my_bytes = 4 * (n + out_n)
+    t = torch.tensor([step_ms, float(my_bytes)], dtype=torch.float64, device=dev)
+    if world > 1:
+        tmax = t[:1].clone()
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        tsum = t[1:].clone()
+        dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
+        step_ms_max, all_bytes = float(tmax.item()), float(tsum.item())
+    else:
+        step_ms_max, all_bytes = step_ms, float(my_bytes)
+    ms_per_step = step_ms_max / args.steps
+    value = all_bytes / (ms_per_step * 1e-3) / 1e9
+
+    # ---- e2e through the public API with host buffers (pinned), copies inside the timing
+    e2e = None
+    if not args.no_e2e:
+        host_in = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        host_in.copy_(pristine)
+        host_out = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        e2e_t = []
+        for i in range(1 + args.e2e_steps):
+            barrier()
+            t0 = time.perf_counter()
+            work.copy_(host_in, non_blocking=True)            # H2D of the step's input
+            res = ds.compact(work, 0, stream)                  # C ABI + NCCL + offsets
+            cnt = int(res.count.item())                        # D2H of the count (syncs)
+            host_out[:cnt].copy_(work[:cnt], non_blocking=True)  # D2H of the result
+            torch.cuda.synchronize()
+            dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+            if world > 1:
+                dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+            if i > 0:
+                e2e_t.append(float(dt.item()))
+        ms_e2e = statistics.median(e2e_t) * 1e3
+        e2e = {"value": round(all_bytes / (ms_e2e * 1e-3) / 1e9, 2), "unit": "GB/s",
+               "h2d_bytes_per_step": 4 * n, "d2h_bytes_per_step": 4 * out_n + 8,
+               "ms_per_step": round(ms_e2e, 2), "steps": args.e2e_steps,
+               "note": "per rank; host->device copy of the shard from pinned memory, ds_compact_ex, "
+                       "count all-gather + ds_shard_offsets, device->host copy of the kept prefix"}
+        del host_in, host_out
+
+    rows = None
+    if rank == 0 and world == 1 and not args.no_rows:
+        del work, pristine
+        torch.cuda.empty_cache()
+        rows = bench_rows(peak, flush)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        n_sample = 1 << 26
+        gbs, t_s, _ = cpu_oracle_sample(n_sample, 3)
+        cpu = {"value": round(gbs, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
+               "sample": f"oracle_compact (sequential C, 1 thread of {os.cpu_count()}) on a "
+                         f"2^26-word sample of the C5 recipe, median of 3 ({t_s * 1e3:.0f} ms each)"}
+
+    if rank == 0:
+        kbytes = 4 * (n + out_n)
+        achieved = kbytes / (kern_ms * 1e-3) / 1e9
+        traffic = load_ncu_traffic()
+        line = {
+            "metric": METRIC, "value": round(value, 1), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+            "dtype": "int32", "data": "synthetic (counter-based hash, dsgen; seeded per global index)",
+            "impl": "libds",
+            "config": {"workload": WORKLOAD, "n_total": N_TOTAL, "n_per_rank": n, "valid_fraction": FRAC,
+                       "out_n": total_out, "parallelism": f"shard{world} (contiguous ranges)",
+                       "l2": "inputs 16/N GiB per rank >> 126 MB L2; L2 also flushed by reading 512 MiB "
+                             "between steps",
+                       "restore": "pristine shard restored by a D2D copy between steps, outside the events",
+                       "step": "ds_compact_ex + NCCL all-gather of counts + ds_shard_offsets"},
+            "frac_of_peak": round(value / world / peak, 4),
+            "elems_per_s": round(N_TOTAL / (ms_per_step * 1e-3), 1),
+            "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                         "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "kernel": "irregular_kernel<OpCompact> (rank 0)", "peak_source": peak_src,
+                         "kernel_ms": round(kern_ms, 4),
+                         "algorithmic_bytes_per_launch": kbytes},
+            "clocks": clk, "gpu_launches": launches,
+        }
+        if e2e:
+            line["e2e"] = e2e
+        if cpu:
+            line["cpu_baseline"] = cpu
+        if rows:
+            line["rows"] = rows
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="libds", choices=["libds", "reference"])
+    ap.add_argument("--no-rows", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "libds" and not os.environ.get("DS_BENCH_ALLOW_SHORT"):
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_libds(args)
+
+
+if __name__ == "__main__":
+    main()
