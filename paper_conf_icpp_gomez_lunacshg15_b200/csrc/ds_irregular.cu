@@ -86,33 +86,47 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 }
 
 // ---- CTA shape ----------------------------------------------------------
-constexpr int kRankWarps = 16;
+#ifndef DS_IRR_RANK_WARPS
+#define DS_IRR_RANK_WARPS 16
+#endif
+#ifndef DS_IRR_IN_STAGES
+#define DS_IRR_IN_STAGES 6
+#endif
+#ifndef DS_IRR_RING_WORDS
+#define DS_IRR_RING_WORDS 0
+#endif
+#ifndef DS_IRR_SLOTS
+#define DS_IRR_SLOTS 16
+#endif
+#ifndef DS_IRR_RESOLVERS
+#define DS_IRR_RESOLVERS 8
+#endif
+constexpr int kRankWarps = DS_IRR_RANK_WARPS;
 constexpr int kRT = 32 * kRankWarps;      // ranker threads
 constexpr int kSeg = 512;                 // contiguous words ranked by one warp
 constexpr int kGroup = 8;                 // contiguous words per lane per group
 constexpr int kGroups = kSeg / (32 * kGroup);  // groups per warp (2)
-constexpr int kT = kRankWarps * kSeg;     // 8192 words = 32 KB per tile
-#ifndef DS_IRR_STAGES
-#define DS_IRR_STAGES 6
-#endif
-constexpr int kResolvers = DS_IRR_STAGES;  // one per stage
+constexpr int kT = kRankWarps * kSeg;     // words per tile (8192 = 32 KB with 16 rankers)
+constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
+constexpr int kRingWords = DS_IRR_RING_WORDS; // compacted tiles awaiting their prefix (0: none)
+constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
+constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
 constexpr int kStoreWarps = 6;
 constexpr int kST = 32 * kStoreWarps;
-constexpr int kWarpResolver0 = kRankWarps;                 // 16..21
-constexpr int kWarpStorer0 = kRankWarps + kResolvers;      // 22..27
-constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;  // 28
+constexpr int kWarpResolver0 = kRankWarps;
+constexpr int kWarpStorer0 = kRankWarps + kResolvers;
+constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;
 constexpr int kThreads = 32 * (kWarpProducer + 1);
 constexpr int kPre = 4;                   // words before the tile (unique's boundary word)
 constexpr int kStageWords = kT + kPre + 4;
-constexpr int kStages = DS_IRR_STAGES;
-#ifndef DS_IRR_MAXLOADS
-#define DS_IRR_MAXLOADS 3
-#endif
-constexpr uint32_t kMaxLoads = DS_IRR_MAXLOADS;  // tile copies in flight per CTA
-constexpr size_t kSmem = size_t(kStages) * kStageWords * 4;
+constexpr size_t kSmem = (size_t(kInStages) * kStageWords + kRingWords) * 4;
 static_assert(kRankWarps <= 32, "warp-total scan in one warp");
-static_assert(kResolvers == kStages, "resolver r serves stage r");
-static_assert(kSmem <= 227 * 1024, "shared memory");
+static_assert(kThreads <= 1024, "CTA size");
+static_assert(kSlots >= kInStages, "a slot per input stage at least");
+static_assert(kSlots % kResolvers == 0, "a slot is always served by the same resolver");
+static_assert(kRingWords % 4 == 0 && (kRingWords == 0 || kRingWords >= kT + 16),
+              "no ring, or a ring that holds one full tile");
+static_assert(kSmem <= 227 * 1024 - 4096, "shared memory");
 
 // Keep mask of the kGroup words w[] at tile word index x (from the staged
 // tile).
@@ -170,6 +184,18 @@ __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) 
 #define DS_IRR_LB 4
 #endif
 constexpr int kLB = DS_IRR_LB;  // look-back slots per lane (32 * kLB tiles per round)
+#ifndef DS_IRR_REFRESH
+#define DS_IRR_REFRESH 1
+#endif
+#ifndef DS_IRR_POLL_MIN
+#define DS_IRR_POLL_MIN 64
+#endif
+#ifndef DS_IRR_POLL_MAX
+#define DS_IRR_POLL_MAX 512
+#endif
+constexpr int kRefreshRows = DS_IRR_REFRESH;        // AGG rows re-read while polling
+constexpr uint32_t kPollMinNs = DS_IRR_POLL_MIN;   // first back-off
+constexpr uint32_t kPollMaxNs = DS_IRR_POLL_MAX;   // back-off cap
 
 __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status, uint32_t tile,
                                              uint32_t epoch, int lane, uint64_t* trace) {
@@ -188,7 +214,7 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status
         for (int m = 0; m < kLB; ++m)
             if (status_current(s[m], epoch)) okm |= 1u << m;
         if (rounds++ == 0 && lane == 0) trace_event(trace, tile, 10, globaltimer());
-        uint32_t ns = 0;
+        uint32_t ns = kPollMinNs;
         uint32_t M, L;  // nearest INCL at slot M, lane L (M == kLB: none this round)
         while (true) {
             uint32_t inclm = 0;
@@ -201,14 +227,23 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status
             const uint32_t need = (M < kLB ? ((1u << M) - 1u) : ((1u << kLB) - 1u)) |
                                   (M < kLB && uint32_t(lane) <= L ? (1u << M) : 0u);
             if (!__any_sync(kFull, (okm & need) != need)) break;
-            if (ns) __nanosleep(ns);
-            ns = ns ? (ns < 256 ? ns * 2 : 256) : 32;
+            __nanosleep(ns);
+            ns = ns < kPollMaxNs ? ns * 2 : kPollMaxNs;
             ++polls;
+            // Re-read the needed slots that are still pending, and refresh the
+            // nearest 32 predecessors even if they hold AGG: a nearer INCL ends the
+            // walk sooner.  Farther AGG slots are not re-read (poll traffic hits
+            // the same few L2 lines from every resolver).
 #pragma unroll
             for (int m = 0; m < kLB; ++m) {
-                if (!(okm >> m & 1u) && (need >> m & 1u)) {
-                    s[m] = ld_relaxed_gpu(status_ptr(status, base - (32 * m + lane)));
-                    if (status_current(s[m], epoch)) okm |= 1u << m;
+                const bool pending = !(okm >> m & 1u);
+                const bool refresh = m < kRefreshRows && !pending && status_state(s[m]) != kStateIncl;
+                if ((need >> m & 1u) && (pending || refresh)) {
+                    const int64_t idx = base - (32 * m + lane);
+                    if (idx >= 0) {
+                        s[m] = ld_relaxed_gpu(status_ptr(status, idx));
+                        okm = status_current(s[m], epoch) ? (okm | 1u << m) : (okm & ~(1u << m));
+                    }
                 }
             }
         }
@@ -237,10 +272,14 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status
     return excl;
 }
 
-struct StageMeta {
-    uint32_t tile;           // kNoTile: end of this CTA's work
-    uint32_t total;          // kept words in the tile
-    unsigned long long excl; // kept words in all lower tiles
+struct SlotMeta {
+    uint32_t tile;              // kNoTile: end of this CTA's work
+    uint32_t total;             // kept words in the tile
+    unsigned long long excl;    // kept words in all lower tiles
+    uint32_t ring_base;         // ring word index of rank 0 (multiple of 4, >= 4)
+    uint32_t ring_end;          // ring allocation counter after this tile
+    uint32_t in_ring;           // compacted into the ring (else in place in its input stage)
+    uint32_t tail_snap;         // ring tail seen before the decision
     uint32_t wtot[kRankWarps];  // kept words in each ranker warp's segment
 };
 
@@ -260,23 +299,30 @@ __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
 template <class Op>
 __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParams p) {
     extern __shared__ __align__(128) uint32_t smem[];
-    __shared__ __align__(8) uint64_t bar_drawn[kStages], bar_full[kStages], bar_counted[kStages], bar_ranked[kStages],
-        bar_resolved[kStages], bar_empty[kStages];
-    __shared__ StageMeta meta[kStages];
+    uint32_t* const ring = smem + kInStages * kStageWords;
+    __shared__ __align__(8) uint64_t bar_full[kInStages], bar_free[kInStages];
+    __shared__ __align__(8) uint64_t bar_drawn[kSlots], bar_counted[kSlots], bar_ranked[kSlots],
+        bar_resolved[kSlots], bar_stored[kSlots];
+    __shared__ SlotMeta meta[kSlots];
     __shared__ uint32_t s_epoch;
-    __shared__ volatile uint32_t s_end;  // ring position of the end marker
+    __shared__ volatile uint32_t s_end;        // ring position of the end marker
+    __shared__ volatile uint32_t s_ring_tail;  // ring words released by the storers (monotone)
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
-        for (int s = 0; s < kStages; ++s) {
-            mbar_init(&bar_drawn[s], 1);
+        for (int s = 0; s < kInStages; ++s) {
             mbar_init(&bar_full[s], 1);
-            mbar_init(&bar_counted[s], 1);
-            mbar_init(&bar_ranked[s], 1);
-            mbar_init(&bar_resolved[s], 1);
-            mbar_init(&bar_empty[s], kStoreWarps);
+            mbar_init(&bar_free[s], 1);
+        }
+        for (int o = 0; o < kSlots; ++o) {
+            mbar_init(&bar_drawn[o], 1);
+            mbar_init(&bar_counted[o], 1);
+            mbar_init(&bar_ranked[o], kRankWarps);
+            mbar_init(&bar_resolved[o], 1);
+            mbar_init(&bar_stored[o], 1);
         }
         s_end = 0xffffffffu;
+        s_ring_tail = 0;
         mbar_fence_init();
     }
     __syncthreads();
@@ -285,28 +331,22 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         // ------------------------------------------------ producer (lane 0)
         if (lane != 0) return;
         for (uint32_t k = 0;; ++k) {
-            const int s = k % kStages;
-            const uint32_t use = k / kStages;
+            const int s = k % kInStages, o = k % kSlots;
             uint32_t* stage = smem + s * kStageWords;
-            mbar_wait(&bar_empty[s], (use & 1) ^ 1);  // storers released tile k - kStages
-            if (k >= kMaxLoads) {
-                // At most kMaxLoads tile copies in flight per CTA: deeper queues only
-                // add latency to the status words' round trips.
-                const uint32_t kp = k - kMaxLoads;
-                mbar_wait(&bar_full[kp % kStages], (kp / kStages) & 1);
-            }
+            mbar_wait(&bar_free[s], ((k / kInStages) & 1) ^ 1);  // rankers hold tile k - kInStages
+            mbar_wait(&bar_stored[o], ((k / kSlots) & 1) ^ 1);   // slot o finished tile k - kSlots
             uint32_t t, epoch;
             draw_ticket(p.ctrl, p.draws, t, epoch);
             if (k == 0) s_epoch = epoch;
             if (t >= p.ntiles) {  // one failed draw per CTA ends its work
-                meta[s].tile = kNoTile;
+                meta[o].tile = kNoTile;
                 s_end = k;
-                mbar_arrive(&bar_drawn[s]);
+                mbar_arrive(&bar_drawn[o]);
                 mbar_arrive(&bar_full[s]);
                 return;
             }
-            meta[s].tile = t;
-            mbar_arrive(&bar_drawn[s]);  // the resolver starts this tile's look-back now
+            meta[o].tile = t;
+            mbar_arrive(&bar_drawn[o]);  // the resolver starts this tile's look-back now
             trace_event(p.trace, t, 0, globaltimer());
             trace_event(p.trace, t, 7, smid());
             debug_delay(t, 0);
@@ -326,16 +366,13 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         bool has_hprev = false;
         uint32_t hprev = 0;
         if (Op::kUnique) has_hprev = halo_prev(p, hprev);
+        uint32_t ring_head = 0;  // output-ring allocation counter (monotone, words; same in every warp)
         for (uint32_t k = 0;; ++k) {
-            const int s = k % kStages;
-            const uint32_t use = k / kStages;
+            const int s = k % kInStages, o = k % kSlots;
             uint32_t* stage = smem + s * kStageWords;
-            mbar_wait(&bar_full[s], use & 1);
-            const uint32_t t = meta[s].tile;
-            if (t == kNoTile) {
-                if (rt == 0) mbar_arrive(&bar_counted[s]);
-                break;
-            }
+            mbar_wait(&bar_full[s], (k / kInStages) & 1);
+            const uint32_t t = meta[o].tile;
+            if (t == kNoTile) break;
             if (rt == 0) trace_event(p.trace, t, 1, globaltimer());
             const uint64_t tb = uint64_t(t) * kT;
             const bool full = tb >= p.lo && tb + kT <= p.hi;
@@ -366,54 +403,75 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 goff |= wrun << (16 * g);
                 wrun += __popc(b0) + 2u * __popc(b1) + 4u * __popc(b2) + 8u * __popc(b3);
             }
-            if (lane == 0) meta[s].wtot[rw] = wrun;
-            named_bar_sync(1, kRT);  // warp totals written; every ranker holds its words
+            if (lane == 0) meta[o].wtot[rw] = wrun;
+            if (rt == 0) meta[o].tail_snap = s_ring_tail;  // the ring tail only grows
+            named_bar_sync(1, kRT);  // warp totals + tail snapshot written; every ranker holds its words
 
             // Exclusive scan of the kRankWarps warp totals (input order), redundantly
             // in every warp.
-            const uint32_t cw = lane < kRankWarps ? meta[s].wtot[lane] : 0u;
+            const uint32_t cw = lane < kRankWarps ? meta[o].wtot[lane] : 0u;
             uint32_t iw = cw;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(kFull, iw, o);
-                if (lane >= o) iw += y;
+            for (int sh = 1; sh < 32; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, iw, sh);
+                if (lane >= sh) iw += y;
             }
             const uint32_t total = __shfl_sync(kFull, iw, 31);
             const uint32_t wbase = __shfl_sync(kFull, iw - cw, rw);
+            // Where to compact: into the output ring if the tile fits against the
+            // tail snapshot (then the input stage is free at once), else in place in
+            // the input stage (the storers free it).  Never waiting here keeps every
+            // drawn tile's AGG independent of other tiles.  Ring allocation:
+            // [4 slack | total rounded up to 4 | 4 slack], contiguous (skip to the
+            // start rather than wrap).  Every warp computes the same decision and
+            // allocation from the same values, so no further barrier is needed.
+            const uint32_t need = 8u + ((total + 3u) & ~3u);
+            const uint32_t pos = kRingWords ? ring_head % kRingWords : 0u;
+            const uint32_t skip = pos + need > uint32_t(kRingWords) ? uint32_t(kRingWords) - pos : 0u;
+            const bool in_ring = kRingWords > 0 && ring_head + skip + need - meta[o].tail_snap <= uint32_t(kRingWords);
+            uint32_t base = kPre;
+            if (in_ring) {
+                base = (ring_head + skip) % (kRingWords ? kRingWords : 1) + 4u;
+                ring_head += skip + need;
+            }
+            if (rt == 0 && in_ring) mbar_arrive(&bar_free[s]);  // the input stage may be refilled
             if (rt == 0) {
                 // a4: publish the aggregate right away -- it depends on nothing else
-                // (a relaxed status store), then hand the total to
-                // this stage's resolver.
-                meta[s].total = total;
+                // (a relaxed status store).
+                meta[o].total = total;
+                meta[o].ring_base = base;
+                meta[o].ring_end = ring_head;
+                meta[o].in_ring = in_ring;
                 debug_delay(t, 1);
                 publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
                 trace_event(p.trace, t, 2, globaltimer());
-                mbar_arrive(&bar_counted[s]);
+                mbar_arrive(&bar_counted[o]);
             }
 
-            // a6: compact the kept words in place: rank r -> stage[kPre + r].
+            // a6: compact the kept words: rank r -> ring[base + r], or in place
+            // -> stage[kPre + r] (every ranker's words are in registers).
+            uint32_t* out = (in_ring ? ring : stage) + base;
 #pragma unroll
             for (int g = 0; g < kGroups; ++g) {
                 uint32_t r = wbase + ((goff >> (16 * g)) & 0xFFFFu) + ((lane_pre >> (16 * g)) & 0xFFFFu);
                 const uint32_t m = masks >> (kGroup * g);
 #pragma unroll
-                for (int k = 0; k < kGroup; ++k)
-                    if (m >> k & 1u) stage[kPre + r++] = v[g][k];
+                for (int kk = 0; kk < kGroup; ++kk)
+                    if (m >> kk & 1u) out[r++] = v[g][kk];
             }
-            named_bar_sync(1, kRT);  // compacted tile complete
-            if (rt == 0) mbar_arrive(&bar_ranked[s]);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is in the ring
         }
     } else if (warp < kWarpStorer0) {
         // ------------------------------------------------ resolver warps
-        // Resolver r serves stage r: ring positions k = r, r + kStages, ...
         const uint32_t r = warp - kWarpResolver0;
-        for (uint32_t k = r;; k += kStages) {
-            const int s = int(r);
-            const uint32_t use = k / kStages;
-            if (!mbar_wait_or_end(&bar_drawn[s], use & 1, &s_end, k)) break;
-            const uint32_t t = meta[s].tile;
+        for (uint32_t k = r;; k += kResolvers) {
+            const int o = k % kSlots;
+            const uint32_t use = k / kSlots;
+            if (!mbar_wait_or_end(&bar_drawn[o], use & 1, &s_end, k)) break;
+            const uint32_t t = meta[o].tile;
             if (t == kNoTile) {
-                if (lane == 0) mbar_arrive(&bar_resolved[s]);
+                if (lane == 0) mbar_arrive(&bar_resolved[o]);
                 break;
             }
             const uint32_t epoch = s_epoch;
@@ -429,37 +487,38 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
 #else
             const uint64_t excl = t > 0 ? lookback(p.status, t, epoch, lane, p.trace) : 0ull;
 #endif
-            mbar_wait(&bar_counted[s], use & 1);  // the tile's aggregate is published
-            const uint32_t total = meta[s].total;
+            mbar_wait(&bar_counted[o], use & 1);  // the tile's aggregate is published
+            const uint32_t total = meta[o].total;
             if (lane == 0 && t > 0)
                 publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
-            mbar_wait(&bar_ranked[s], use & 1);  // the compacted tile is in the stage
+            mbar_wait(&bar_ranked[o], use & 1);  // the compacted tile is in the ring
             if (lane == 0) {
                 trace_event(p.trace, t, 4, globaltimer());
-                meta[s].excl = excl;
+                meta[o].excl = excl;
                 if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = excl + total;
-                mbar_arrive(&bar_resolved[s]);
+                mbar_arrive(&bar_resolved[o]);
             }
         }
     } else {
         // ------------------------------------------------ storer warps
         const int st = tid - 32 * kWarpStorer0;
         for (uint32_t k = 0;; ++k) {
-            const int s = k % kStages;
-            const uint32_t use = k / kStages;
-            const uint32_t* stage = smem + s * kStageWords;
-            mbar_wait(&bar_resolved[s], use & 1);
-            const uint32_t t = meta[s].tile;
+            const int o = k % kSlots;
+            mbar_wait(&bar_resolved[o], (k / kSlots) & 1);
+            const uint32_t t = meta[o].tile;
             if (t == kNoTile) break;
             if (st == 0) {
                 trace_event(p.trace, t, 5, globaltimer());
                 debug_delay(t, 3);
             }
             // a7: chunk c covers virtual words c0 + 4c + [0, 4) = ranks 4c - ph + [0, 4)
-            // (ph = 16-byte phase of the output start), read from the stage as
-            // two aligned vectors and funnel-shifted.
-            const uint32_t A = meta[s].total;
-            const uint64_t s0 = p.lo + meta[s].excl;
+            // (ph = 16-byte phase of the output start), read as two aligned vectors
+            // of the ring and funnel-shifted.
+            const bool in_ring = meta[o].in_ring != 0;
+            const int s_in = k % kInStages;
+            const uint32_t* src = (in_ring ? ring : smem + s_in * kStageWords) + meta[o].ring_base;
+            const uint32_t A = meta[o].total;
+            const uint64_t s0 = p.lo + meta[o].excl;
             const uint64_t s1 = s0 + A;
             const uint64_t c0 = s0 & ~3ull;
             const uint32_t ph = uint32_t(s0 & 3);
@@ -468,29 +527,46 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
 #else
             const uint32_t nchunks = A ? uint32_t((s1 - c0 + 3) >> 2) : 0u;
 #endif
-            for (uint32_t c = st; c < nchunks; c += kST) {
-                const u32x4 hi = *reinterpret_cast<const u32x4*>(stage + kPre + 4 * c);
-                const u32x4 lo = *reinterpret_cast<const u32x4*>(stage + kPre + 4 * c - 4);
-                uint32_t w0, w1, w2, w3;
-                switch (ph) {  // warp-uniform
-                case 0: w0 = hi.x; w1 = hi.y; w2 = hi.z; w3 = hi.w; break;
-                case 1: w0 = lo.w; w1 = hi.x; w2 = hi.y; w3 = hi.z; break;
-                case 2: w0 = lo.z; w1 = lo.w; w2 = hi.x; w3 = hi.y; break;
-                default: w0 = lo.y; w1 = lo.z; w2 = lo.w; w3 = hi.x; break;
-                }
-                const uint64_t g = c0 + 4ull * c;
-                if (g >= s0 && g + 4 <= s1) {
-                    stg_stream_v4(p.abase + g, w0, w1, w2, w3);
-                } else {
-                    const uint32_t w[4] = {w0, w1, w2, w3};
+            // Four chunks per thread per iteration: all shared loads first, then the
+            // global stores (ILP).
+            constexpr int kU = 4;
+            for (uint32_t c0i = st; c0i < nchunks; c0i += kU * kST) {
+                uint32_t w[kU][4];
 #pragma unroll
-                    for (int kk = 0; kk < 4; ++kk)
-                        if (g + kk >= s0 && g + kk < s1) stg_stream(p.abase + g + kk, w[kk]);
+                for (int u = 0; u < kU; ++u) {
+                    const uint32_t c = c0i + u * kST;
+                    if (c < nchunks) {
+                        const u32x4 hi = *reinterpret_cast<const u32x4*>(src + 4 * c);
+                        const u32x4 lo = *reinterpret_cast<const u32x4*>(src + 4 * c - 4);
+                        switch (ph) {  // warp-uniform
+                        case 0: w[u][0] = hi.x; w[u][1] = hi.y; w[u][2] = hi.z; w[u][3] = hi.w; break;
+                        case 1: w[u][0] = lo.w; w[u][1] = hi.x; w[u][2] = hi.y; w[u][3] = hi.z; break;
+                        case 2: w[u][0] = lo.z; w[u][1] = lo.w; w[u][2] = hi.x; w[u][3] = hi.y; break;
+                        default: w[u][0] = lo.y; w[u][1] = lo.z; w[u][2] = lo.w; w[u][3] = hi.x; break;
+                        }
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < kU; ++u) {
+                    const uint32_t c = c0i + u * kST;
+                    if (c >= nchunks) break;
+                    const uint64_t g = c0 + 4ull * c;
+                    if (g >= s0 && g + 4 <= s1) {
+                        stg_stream_v4(p.abase + g, w[u][0], w[u][1], w[u][2], w[u][3]);
+                    } else {
+#pragma unroll
+                        for (int kk = 0; kk < 4; ++kk)
+                            if (g + kk >= s0 && g + kk < s1) stg_stream(p.abase + g + kk, w[u][kk]);
+                    }
                 }
             }
-            __syncwarp();
-            if (st == 0) trace_event(p.trace, t, 6, globaltimer());
-            if (lane == 0) mbar_arrive(&bar_empty[s]);  // this warp is done with the stage
+            named_bar_sync(2, kST);  // every storer is done reading the tile's ring space
+            if (st == 0) {
+                trace_event(p.trace, t, 6, globaltimer());
+                if (in_ring) s_ring_tail = meta[o].ring_end;
+                else mbar_arrive(&bar_free[s_in]);  // the in-place tile's input stage is free
+                mbar_arrive(&bar_stored[o]);
+            }
         }
     }
 }

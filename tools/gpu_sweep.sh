@@ -1,6 +1,4 @@
 mkdir -p gpurun_out
-timeout 600 python -m pytest tests -m "gpu and not slow" -x -q --timeout 120 --timeout-method thread > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
-tail -3 gpurun_out/pytest_gpu.log
-for v in libds libds_lb4; do
-  echo "== $v"; LIBDS_PATH=$PWD/paper_conf_icpp_gomez_lunacshg15_b200/lib/$v.so timeout 120 python tools/trace_pipeline.py 30 0.5 2>&1 | grep -E "rate|lb:first|lb:resolve|^load|^count|^lookback|wait-for|incl-after|cwait|polls|consume"
-done 2>&1 | tee gpurun_out/sweep.log
+for v in p1_64_512_st4 p0_64_512_st4 p4_32_256_st4 p1_128_1024_st4 p1_64_512_st1 p1_64_512_st2; do for f in 0.1 0.5 0.9; do
+  echo "== $v f=$f"; LIBDS_PATH=$PWD/paper_conf_icpp_gomez_lunacshg15_b200/lib/libds_$v.so timeout 120 python tools/trace_pipeline.py 30 $f 2>&1 | grep -E "rate|polls"
+done; done 2>&1 | tee gpurun_out/sweep.log

@@ -20,7 +20,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import dsgen  # noqa: E402
 from paper_conf_icpp_gomez_lunacshg15_b200 import libds  # noqa: E402
 
-T = 8192
+T = int(os.environ.get("DS_TILE", "8192"))
 
 
 def main():
