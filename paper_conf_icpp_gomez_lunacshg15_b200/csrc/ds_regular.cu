@@ -50,6 +50,7 @@ struct RegParams {
     uint32_t draws;   // ntiles + gridDim.x
     uint64_t* status;
     uint64_t* ctrl;
+    uint64_t* trace;  // diagnostics: per-tile events, or null
 };
 
 struct TileGeom {
@@ -157,7 +158,7 @@ constexpr int kVec = kItems / 4;
 constexpr int kT = kCT * kItems;          // 8192 output words = 32 KB per tile
 constexpr int kStageWords = kT + 512;     // staged source span cap (words)
 constexpr int kStages = 3;
-constexpr int kThreads = 32 * (1 + kConsumerWarps);
+constexpr int kThreads = 32 * (2 + kConsumerWarps);  // producer, publisher, consumers
 constexpr size_t kSmem = size_t(kStages) * kStageWords * 4;
 
 struct StageMeta {
@@ -215,7 +216,8 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
 
     if (warp == 0) {
         // ------------------------------------------------ producer warp
-        // r1 draw, r2 load, r3a publish LOADED as soon as the sources landed.
+        // r1 draw + geometry, r2 start the tile's source copy; up to kStages
+        // copies in flight (the publisher warp waits for them).
         for (uint32_t k = 0;; ++k) {
             const int s = k % kStages;
             const uint32_t use = k / kStages;
@@ -228,12 +230,14 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
             if (t >= p.ntiles) {  // one failed draw per CTA ends its work
                 if (lane == 0) {
                     meta[s].g.k = kNoTile;
-                    mbar_arrive(&bar_loaded[s]);
+                    mbar_arrive(&bar_full[s]);
                 }
                 break;
             }
             const int64_t kt = PAD ? int64_t(p.ntiles) - 1 - t : int64_t(t);
             if (lane == 0) {
+                trace_event(p.trace, uint64_t(kt), 0, globaltimer());
+                trace_event(p.trace, uint64_t(kt), 7, smid());
                 debug_delay(uint64_t(kt), 0);
                 tile_geometry<PAD, kT, kStageWords>(p, kt, meta[s].g);
                 meta[s].epoch = epoch;
@@ -251,16 +255,29 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
                 if (g.span > 0) gather_slow<PAD>(p, g, stage, lane);
                 if (lane == 0) mbar_arrive(&bar_full[s]);
             }
+        }
+    } else if (warp == 1) {
+        // ------------------------------------------------ publisher warp
+        // r3a: publish LOADED as soon as each tile's sources landed, in order.
+        for (uint32_t k = 0;; ++k) {
+            const int s = k % kStages;
+            const uint32_t use = k / kStages;
             mbar_wait(&bar_full[s], use & 1);
+            const int64_t kt = meta[s].g.k;
             if (lane == 0) {
-                debug_delay(uint64_t(kt), 1);
-                publish_status(status_ptr(p.status, kt), make_status(kStateLoaded, epoch, 0));
+                if (kt != kNoTile) {
+                    trace_event(p.trace, uint64_t(kt), 1, globaltimer());
+                    debug_delay(uint64_t(kt), 1);
+                    publish_status(status_ptr(p.status, kt), make_status(kStateLoaded, meta[s].epoch, 0));
+                    trace_event(p.trace, uint64_t(kt), 2, globaltimer());
+                }
                 mbar_arrive(&bar_loaded[s]);
             }
+            if (kt == kNoTile) break;
         }
     } else {
         // ------------------------------------------------ consumer warps
-        const int ct = tid - 32;
+        const int ct = tid - 64;
         for (uint32_t k = 0;; ++k) {
             const int s = k % kStages;
             const uint32_t use = k / kStages;
@@ -272,12 +289,16 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
 
             // r3b: the first consumer warp waits for the earlier-ticketed tiles
             // whose sources lie in this tile's output range ...
-            if (warp == 1 && g.win_lo <= g.win_hi)
-                wait_loaded(p.status, g.win_lo, g.win_hi, meta[s].epoch, lane);
+            if (warp == 2) {
+                if (lane == 0) trace_event(p.trace, uint64_t(g.k), 3, globaltimer());
+                if (g.win_lo <= g.win_hi) wait_loaded(p.status, g.win_lo, g.win_hi, meta[s].epoch, lane);
+                if (lane == 0) trace_event(p.trace, uint64_t(g.k), 4, globaltimer());
+            }
 
             // ... while every consumer gathers its outputs (r4).
             uint32_t o[kVec][4];
             const int32_t soff = int32_t(g.slo + mis - g.sb);
+            const uint32_t data_cols = PAD ? p.Cw : p.NCw;  // columns that carry source words
 #pragma unroll
             for (int i = 0; i < kVec; ++i) {
                 const int64_t vq = V0 + 4 * int64_t(i * kCT + ct) - mis;  // output word of slot 0
@@ -285,6 +306,29 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
                 uint32_t t = uint32_t(xq) + g.col0;  // only meaningful when vq >= q0
                 uint32_t dr = fastdiv(t, p.div_nc);
                 uint32_t col = t - dr * p.NCw;
+                const bool whole = vq >= g.q0 && vq + 4 <= g.q1;
+                if (whole && g.bytes && col + 4 <= data_cols) {
+                    // Fast path: four data words of one row segment = four consecutive
+                    // staged source words; two aligned 16-byte shared loads and a
+                    // funnel shift by the segment's phase.
+                    const int32_t sidx = g.base_rel + int32_t(dr * p.Cw + col) + soff;
+                    const uint32_t ph = uint32_t(sidx) & 3u;
+                    const u32x4 A = *reinterpret_cast<const u32x4*>(stage + (sidx & ~3));
+                    const u32x4 B = ph ? *reinterpret_cast<const u32x4*>(stage + (sidx & ~3) + 4) : A;
+                    const bool b0 = ph & 1u, b1 = ph & 2u;
+                    const uint32_t h0 = b0 ? A.y : A.x, h1 = b0 ? A.z : A.y, h2 = b0 ? A.w : A.z;
+                    const uint32_t h3 = b0 ? B.x : A.w, h4 = b0 ? B.y : B.x, h5 = b0 ? B.z : B.y;
+                    o[i][0] = b1 ? h2 : h0;
+                    o[i][1] = b1 ? h3 : h1;
+                    o[i][2] = b1 ? h4 : h2;
+                    o[i][3] = b1 ? h5 : h3;
+                    continue;
+                }
+                if (PAD && whole && col >= p.Cw && col + 4 <= p.NCw) {  // four fill cells
+#pragma unroll
+                    for (int kk = 0; kk < 4; ++kk) o[i][kk] = fill_word(p, col + kk);
+                    continue;
+                }
 #pragma unroll
                 for (int kk = 0; kk < 4; ++kk) {
                     const int64_t q = vq + kk;
@@ -314,6 +358,7 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
             if (lane == 0) mbar_arrive(&bar_empty[s]);  // this warp is done with the stage
             if (ct == 0) debug_delay(uint64_t(g.k), 2);
             named_bar_sync(1, kCT);  // the window wait (acquire fence) precedes every store
+            if (ct == 0) trace_event(p.trace, uint64_t(g.k), 5, globaltimer());
 
             // r5: store stage.
 #pragma unroll
@@ -329,6 +374,7 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
                             stg_stream(p.abase + u + kk, o[i][kk]);
                 }
             }
+            if (ct == 0) trace_event(p.trace, uint64_t(g.k), 6, globaltimer());
         }
     }
 }
@@ -388,6 +434,7 @@ cudaError_t launch_regular(const RegArgs& a, Workspace& ws, cudaStream_t s) {
     p.ntiles = uint32_t(regular_tiles(a));
     p.status = ws.status;
     p.ctrl = ws.ctrl;
+    p.trace = debug_trace(p.ntiles);
     count_launch();
     return a.pad ? launch_dir<true>(p, s) : launch_dir<false>(p, s);
 }
