@@ -55,6 +55,10 @@ def lib():
         L.oracle_unique.restype = sz
         L.oracle_unique_prev.argtypes = [vp, sz, i32, u32]
         L.oracle_unique_prev.restype = sz
+        L.oracle_partition.argtypes = [vp, sz, i32, u32, vp]
+        L.oracle_partition.restype = sz
+        L.oracle_select_copy.argtypes = [vp, sz, i32, u32, vp]
+        L.oracle_select_copy.restype = sz
         L.oracle_pad.argtypes = [vp, sz, sz, sz, sz, vp]
         L.oracle_pad.restype = i32
         L.oracle_unpad.argtypes = [vp, sz, sz, sz, sz]
@@ -99,6 +103,26 @@ def unique(a: np.ndarray, prev: int | None = None) -> int:
     if prev is None:
         return int(lib().oracle_unique(_ptr(a), a.size))
     return int(lib().oracle_unique_prev(_ptr(a), a.size, 1, int(prev) & 0xFFFFFFFF))
+
+
+def partition(a: np.ndarray, pred: int, param: int = 0) -> int:
+    """In place; true words first, then false words, both stable."""
+    a = _words(a)
+    aux = np.empty_like(a)
+    r = lib().oracle_partition(_ptr(a), a.size, int(pred), int(param) & 0xFFFFFFFF, _ptr(aux))
+    if r == ctypes.c_size_t(-1).value:
+        raise ValueError(f"unknown predicate id {pred}")
+    return int(r)
+
+
+def select_copy(a: np.ndarray, pred: int, param: int = 0) -> np.ndarray:
+    """Out of place (P:242 Copy_if): returns the predicate-true words."""
+    a = np.ascontiguousarray(a)
+    out = np.empty(a.size, dtype=np.uint32)
+    r = lib().oracle_select_copy(_ptr(a), a.size, int(pred), int(param) & 0xFFFFFFFF, _ptr(out))
+    if r == ctypes.c_size_t(-1).value:
+        raise ValueError(f"unknown predicate id {pred}")
+    return out[:r].copy()
 
 
 def _bytes_view(buf: np.ndarray) -> np.ndarray:

@@ -73,6 +73,31 @@ size_t oracle_unique(uint32_t* a, size_t n) {
     return oracle_unique_prev(a, n, 0, 0u);
 }
 
+/* P:286-292 partition: true words first, then false words, both in input
+ * order.  The false words go to aux (the paper's Array_false) and are
+ * copied back to the tail "once the true elements have been shifted".     */
+size_t oracle_partition(uint32_t* a, size_t n, int pred, uint32_t param, uint32_t* aux) {
+    if (pred < 0 || pred >= ORACLE_PRED_COUNT) return (size_t)-1;
+    size_t t = 0, f = 0;
+    for (size_t i = 0; i < n; ++i) {
+        uint32_t x = a[i];
+        if (oracle_predicate(pred, x, param)) a[t++] = x;
+        else aux[f++] = x;
+    }
+    for (size_t j = 0; j < f; ++j) a[t + j] = aux[j];
+    return t;
+}
+
+/* P:242 DS Copy_if: out-of-place select. */
+size_t oracle_select_copy(const uint32_t* in, size_t n, int pred, uint32_t param,
+                          uint32_t* out) {
+    if (pred < 0 || pred >= ORACLE_PRED_COUNT) return (size_t)-1;
+    size_t w = 0;
+    for (size_t i = 0; i < n; ++i)
+        if (oracle_predicate(pred, in[i], param)) out[w++] = in[i];
+    return w;
+}
+
 /* "move each row starting from the last one"; row r goes from byte
  * offset r*cols*eb to r*new_cols*eb (a shift of (new_cols-cols)*r elements,
  * "row i will be shifted by C x i"), then its new cells get the fill.    */

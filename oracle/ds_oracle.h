@@ -70,6 +70,19 @@ size_t oracle_unique(uint32_t* a, size_t n);
  * word 0 is compared with `prev` when has_prev != 0, else it is kept.    */
 size_t oracle_unique_prev(uint32_t* a, size_t n, int has_prev, uint32_t prev);
 
+/* Partition: "The elements that satisfy the predicate are
+ * placed in the first part of the array, preceding the elements that do not
+ * satisfy the predicate"; stable for both classes (the DS stability of P:15;
+ * the paper compares with thrust::stable_partition).  In place on a;
+ * `aux` (n words) plays the paper's auxiliary Array_false.  Returns the
+ * number of true words, or (size_t)-1 for an unknown predicate.           */
+size_t oracle_partition(uint32_t* a, size_t n, int pred, uint32_t param, uint32_t* aux);
+
+/* Out-of-place select ("DS Copy_if"): the predicate-true words
+ * of in[0, n) are written in order to out; in is not modified.           */
+size_t oracle_select_copy(const uint32_t* in, size_t n, int pred, uint32_t param,
+                          uint32_t* out);
+
 /* Padding: rows x cols matrix (row-major, elem_bytes per element)
  * at b; the buffer has room for rows x new_cols elements ("the extra memory
  * space needs to be previously allocated adjacent to the matrix").

@@ -163,6 +163,38 @@ def test_select_unknown_predicate():
     assert list(a) == [0, 1, 2, 3, 4]
 
 
+# ------------------------------------------------------------------ partition
+def test_partition_brute_force_all_masks():
+    """Every mask for n <= 9 on index-tagged data (odd tag = true under I32_ODD):
+    trues in order, then falses in order (stable)."""
+    for n in range(0, 10):
+        for mask in range(1 << n):
+            a = np.array([2 * i + 1 if (mask >> i) & 1 else 2 * i + 2 for i in range(n)], dtype=np.uint32)
+            orig = list(a)
+            m = oracle.partition(a, oracle.PRED_I32_ODD)
+            t = [x for x in orig if x % 2 == 1]
+            f = [x for x in orig if x % 2 == 0]
+            assert m == len(t) and list(a) == t + f
+
+
+@pytest.mark.parametrize("pred", range(oracle.PRED_COUNT))
+def test_partition_equals_numpy_concat(pred):
+    a = dsgen.random_words(20011, 300 + pred).numpy().view(np.uint32).copy()
+    keep = _numpy_pred(pred, a, 0x3F800000)
+    x = a.copy()
+    m = oracle.partition(x, pred, 0x3F800000)
+    assert m == int(keep.sum())
+    assert np.array_equal(x, np.concatenate([a[keep], a[~keep]]))  # numpy masking + concatenate
+
+
+def test_select_copy_equals_numpy_and_leaves_input():
+    a = dsgen.random_words(10007, 9).numpy().view(np.uint32).copy()
+    b = a.copy()
+    out = oracle.select_copy(a, oracle.PRED_I32_EVEN)
+    assert np.array_equal(a, b)
+    assert np.array_equal(out, a[(a & 1) == 0])
+
+
 # --------------------------------------------------------------------- unique
 def test_unique_brute_force_small_alphabet():
     """All sequences over {0,1,2} up to length 7 vs itertools.groupby."""
