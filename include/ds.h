@@ -128,6 +128,36 @@ ds_status ds_unique_ex(void* ptr, size_t n, const uint64_t* d_halo,
                        size_t halo_len, uint64_t* d_out_n, ds_stream_t stream);
 
 /* ---------------------------------------------------------------------
+ * Partition and out-of-place variants
+ * ------------------------------------------------------------------- */
+
+/* ds_partition -- stable partition: predicate-true words first,
+ * then the false words, both in input order.  As in the paper, the false
+ * words go through an auxiliary buffer ("Array_false should be an
+ * auxiliary buffer"): `aux` is a caller-owned DEVICE buffer of at
+ * least n words; libds allocates nothing n-sized.  One DS pass slides the
+ * trues in place and writes the falses to aux in order, then a copy moves
+ * them to the tail ptr[*out_n_true, n).  out_n_true: HOST, required.      */
+ds_status ds_partition(void* ptr, size_t n, int predicate_id, void* aux, size_t* out_n_true);
+/* Asynchronous form; d_out_n_true (DEVICE, required) receives the true count. */
+ds_status ds_partition_ex(void* ptr, size_t n, int predicate_id, uint32_t param, void* aux,
+                          uint64_t* d_out_n_true, ds_stream_t stream);
+
+/* ds_select_copy_ex -- out-of-place select ("DS Copy_if"):
+ * the predicate-true words of in[0, n) are written in order to out[0, count);
+ * in is not modified.  out == in gives the in-place select; otherwise the
+ * two buffers must not overlap.                                          */
+ds_status ds_select_copy_ex(const void* in, size_t n, int predicate_id, uint32_t param,
+                            void* out, uint64_t* d_out_n, ds_stream_t stream);
+
+/* ds_partition_copy_ex -- out-of-place stable partition: trues to
+ * out_true[0, t), falses to out_false[0, n - t); in is not modified; the
+ * three buffers must not overlap.  d_out_n_true: DEVICE, may be NULL.    */
+ds_status ds_partition_copy_ex(const void* in, size_t n, int predicate_id, uint32_t param,
+                               void* out_true, void* out_false, uint64_t* d_out_n_true,
+                               ds_stream_t stream);
+
+/* ---------------------------------------------------------------------
  * Sharding helpers (multi-GPU).  Each GPU slides its
  * own contiguous shard; NCCL all-gathers 8-byte values between the calls.
  * ------------------------------------------------------------------- */

@@ -265,6 +265,89 @@ ds_status ds_unique(void* ptr, size_t n, size_t* out_n) {
     return irregular_blocking(a, out_n);
 }
 
+ds_status ds_select_copy_ex(const void* in, size_t n, int predicate_id, uint32_t param, void* out,
+                            uint64_t* d_out_n, ds_stream_t stream) {
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(in, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    if (n > 0 && (!out || misaligned(out, 4))) return DS_ERROR_INVALID_VALUE;
+    ds::IrregArgs a{const_cast<uint32_t*>(static_cast<const uint32_t*>(in)), n, ds::IrregOp::Select,
+                    predicate_id, param, nullptr, 0, d_out_n};
+    a.out_true = static_cast<uint32_t*>(out);
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_partition_copy_ex(const void* in, size_t n, int predicate_id, uint32_t param,
+                               void* out_true, void* out_false, uint64_t* d_out_n_true,
+                               ds_stream_t stream) {
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(in, n, d_out_n_true);
+    if (st != DS_SUCCESS) return st;
+    if (n > 0 && (!out_true || !out_false || misaligned(out_true, 4) || misaligned(out_false, 4)))
+        return DS_ERROR_INVALID_VALUE;
+    ds::IrregArgs a{const_cast<uint32_t*>(static_cast<const uint32_t*>(in)), n, ds::IrregOp::Select,
+                    predicate_id, param, nullptr, 0, d_out_n_true};
+    a.out_true = static_cast<uint32_t*>(out_true);
+    a.out_false = static_cast<uint32_t*>(out_false);
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_partition_ex(void* ptr, size_t n, int predicate_id, uint32_t param, void* aux,
+                          uint64_t* d_out_n_true, ds_stream_t stream) {
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    if (!d_out_n_true) return DS_ERROR_INVALID_VALUE;  // the tail copy needs the true count
+    ds_status st = check_irregular(ptr, n, d_out_n_true);
+    if (st != DS_SUCCESS) return st;
+    if (n > 0 && (!aux || misaligned(aux, 4))) return DS_ERROR_INVALID_VALUE;
+    if (n == 0) return irregular_ex(ds::IrregArgs{static_cast<uint32_t*>(ptr), 0, ds::IrregOp::Select,
+                                                  predicate_id, param, nullptr, 0, d_out_n_true},
+                                    reinterpret_cast<cudaStream_t>(stream));
+    // Step 1 (one DS pass): trues slide in place, falses go to aux in order.
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Select, predicate_id, param,
+                    nullptr, 0, d_out_n_true};
+    a.out_false = static_cast<uint32_t*>(aux);
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    st = run_irregular(a, s);
+    if (st != DS_SUCCESS) return st;
+    // Step 2: aux[0, n - n_true) -> ptr[n_true, n).
+    cudaError_t e = ds::launch_tail_copy(static_cast<uint32_t*>(ptr), d_out_n_true,
+                                         static_cast<const uint32_t*>(aux), nullptr, n, s);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "tail copy launch");
+}
+
+ds_status ds_partition(void* ptr, size_t n, int predicate_id, void* aux, size_t* out_n_true) {
+    if (!out_n_true) return DS_ERROR_INVALID_VALUE;
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(ptr, n, nullptr);
+    if (st != DS_SUCCESS) return st;
+    if (n > 0 && (!aux || misaligned(aux, 4))) return DS_ERROR_INVALID_VALUE;
+    if (n == 0) {
+        *out_n_true = 0;
+        return DS_SUCCESS;
+    }
+    uint64_t* d_cnt = nullptr;
+    uint64_t* h_cnt = nullptr;
+    {
+        std::lock_guard<std::mutex> lock(g_mu);
+        ds::Workspace* ws = nullptr;
+        st = get_workspace(ds::irregular_tiles(ds::IrregArgs{static_cast<uint32_t*>(ptr), n,
+                                                             ds::IrregOp::Select, 0, 0, nullptr, 0, nullptr}),
+                           nullptr, &ws);
+        if (st != DS_SUCCESS) return st;
+        ws->launches--;  // only reserving the count words here
+        d_cnt = ws->d_count;
+        h_cnt = ws->h_count;
+    }
+    st = ds_partition_ex(ptr, n, predicate_id, 0u, aux, d_cnt, nullptr);
+    if (st != DS_SUCCESS) return st;
+    std::lock_guard<std::mutex> lock(g_mu);
+    cudaError_t e = cudaMemcpyAsync(h_cnt, d_cnt, sizeof(uint64_t), cudaMemcpyDeviceToHost, nullptr);
+    if (e != cudaSuccess) return fail(e, "cudaMemcpyAsync");
+    if ((e = cudaStreamSynchronize(nullptr)) != cudaSuccess) return fail(e, "cudaStreamSynchronize");
+    *out_n_true = size_t(*h_cnt);
+    return DS_SUCCESS;
+}
+
 ds_status ds_halo_entry(const void* ptr, size_t n, uint64_t* d_entry, ds_stream_t stream) {
     if (!d_entry || misaligned(d_entry, 8)) return DS_ERROR_INVALID_VALUE;
     if (n > 0 && (ptr == nullptr || misaligned(ptr, 4))) return DS_ERROR_INVALID_VALUE;

@@ -30,6 +30,8 @@ struct IrregArgs {
     const uint64_t* halo;  // Unique
     size_t halo_len;
     uint64_t* d_out_n;  // may be null
+    uint32_t* out_true = nullptr;   // kept / true words (null: in place at ptr)
+    uint32_t* out_false = nullptr;  // false words in input order (null: dropped)
 };
 
 struct RegArgs {
@@ -49,6 +51,9 @@ size_t regular_tiles(const RegArgs& a);
 // Enqueue the kernels; return the cudaError_t of the launch.
 cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s);
 cudaError_t launch_regular(const RegArgs& a, Workspace& ws, cudaStream_t s);
+// Copies n words src[0, n) -> dst_base[*d_offset + j] (partition's tail move).
+cudaError_t launch_tail_copy(uint32_t* dst_base, const uint64_t* d_offset, const uint32_t* src,
+                             const uint64_t* d_count_false, size_t n_total, cudaStream_t s);
 cudaError_t launch_halo_entry(const uint32_t* ptr, size_t n, uint64_t* d_entry, cudaStream_t s);
 cudaError_t launch_shard_offsets(const uint64_t* d_counts, size_t world, size_t rank,
                                  uint64_t* d_result, cudaStream_t s);

@@ -53,7 +53,11 @@ struct IrregParams {
     uint32_t ntiles;
     uint32_t draws;   // ntiles + gridDim.x
     uint32_t value;   // compact: remove value; select: predicate parameter
-    uint64_t* trace;  // diagnostics: 8 timestamps per tile, or null
+    uint64_t* trace;  // diagnostics: per-tile events, or null
+    uint32_t* tbase;  // 16-byte-aligned base of the true/kept output (== abase in place)
+    uint64_t tlo;     // its word offset (output word j lives at tbase[tlo + j])
+    uint32_t* fbase;  // same for the false words (partition), or null
+    uint64_t flo;
 };
 
 // ---- predicates (a3) ----------------------------------------------------
@@ -96,10 +100,10 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 #define DS_IRR_RING_WORDS 0
 #endif
 #ifndef DS_IRR_SLOTS
-#define DS_IRR_SLOTS 16
+#define DS_IRR_SLOTS 12
 #endif
 #ifndef DS_IRR_RESOLVERS
-#define DS_IRR_RESOLVERS 8
+#define DS_IRR_RESOLVERS 6
 #endif
 constexpr int kRankWarps = DS_IRR_RANK_WARPS;
 constexpr int kRT = 32 * kRankWarps;      // ranker threads
@@ -111,7 +115,7 @@ constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
 constexpr int kRingWords = DS_IRR_RING_WORDS; // compacted tiles awaiting their prefix (0: none)
 constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
 constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
-constexpr int kStoreWarps = 6;
+constexpr int kStoreWarps = 5;
 constexpr int kST = 32 * kStoreWarps;
 constexpr int kWarpResolver0 = kRankWarps;
 constexpr int kWarpStorer0 = kRankWarps + kResolvers;
@@ -272,6 +276,56 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status
     return excl;
 }
 
+// a7 helper: write the `cnt` words stage[src_off, src_off + cnt) to the
+// output words base[d0, d0 + cnt) (virtual indices; base is 16-byte aligned).
+// Destination chunks of 4 aligned words are read as two aligned shared
+// vectors and funnel-shifted (the phase is uniform over the segment); whole
+// chunks use one STG.128, the head and tail chunks are written word by word
+// so no word outside the segment is touched.  kSTT threads, 4 chunks per
+// iteration for ILP.
+template <int kSTT>
+__device__ __forceinline__ void store_segment(uint32_t* base, uint64_t d0, uint32_t cnt,
+                                              const uint32_t* stage, int32_t src_off, int st) {
+    if (cnt == 0) return;
+    const uint64_t d1 = d0 + cnt;
+    const uint64_t c0 = d0 & ~3ull;
+    const int32_t bidx = src_off - int32_t(d0 & 3);  // stage index of chunk 0's first word
+    const uint32_t ph = uint32_t(bidx) & 3u;
+    const uint32_t* sv = stage + (bidx & ~3);
+    const uint32_t nchunks = uint32_t((d1 - c0 + 3) >> 2);
+    constexpr int kU = 4;
+    for (uint32_t c0i = st; c0i < nchunks; c0i += kU * kSTT) {
+        uint32_t w[kU][4];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const uint32_t c = c0i + u * kSTT;
+            if (c < nchunks) {
+                const u32x4 lo = *reinterpret_cast<const u32x4*>(sv + 4 * c);
+                const u32x4 hi = ph ? *reinterpret_cast<const u32x4*>(sv + 4 * c + 4) : lo;
+                switch (ph) {  // warp-uniform
+                case 0: w[u][0] = lo.x; w[u][1] = lo.y; w[u][2] = lo.z; w[u][3] = lo.w; break;
+                case 1: w[u][0] = lo.y; w[u][1] = lo.z; w[u][2] = lo.w; w[u][3] = hi.x; break;
+                case 2: w[u][0] = lo.z; w[u][1] = lo.w; w[u][2] = hi.x; w[u][3] = hi.y; break;
+                default: w[u][0] = lo.w; w[u][1] = hi.x; w[u][2] = hi.y; w[u][3] = hi.z; break;
+                }
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const uint32_t c = c0i + u * kSTT;
+            if (c >= nchunks) break;
+            const uint64_t g = c0 + 4ull * c;
+            if (g >= d0 && g + 4 <= d1) {
+                stg_stream_v4(base + g, w[u][0], w[u][1], w[u][2], w[u][3]);
+            } else {
+#pragma unroll
+                for (int kk = 0; kk < 4; ++kk)
+                    if (g + kk >= d0 && g + kk < d1) stg_stream(base + g + kk, w[u][kk]);
+            }
+        }
+    }
+}
+
 struct SlotMeta {
     uint32_t tile;              // kNoTile: end of this CTA's work
     uint32_t total;             // kept words in the tile
@@ -296,7 +350,7 @@ __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
     }
 }
 
-template <class Op>
+template <class Op, bool PART>
 __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParams p) {
     extern __shared__ __align__(128) uint32_t smem[];
     uint32_t* const ring = smem + kInStages * kStageWords;
@@ -428,7 +482,9 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint32_t need = 8u + ((total + 3u) & ~3u);
             const uint32_t pos = kRingWords ? ring_head % kRingWords : 0u;
             const uint32_t skip = pos + need > uint32_t(kRingWords) ? uint32_t(kRingWords) - pos : 0u;
-            const bool in_ring = kRingWords > 0 && ring_head + skip + need - meta[o].tail_snap <= uint32_t(kRingWords);
+            // (partition keeps the whole tile -- trues, then falses -- in its stage)
+            const bool in_ring = !PART && kRingWords > 0 &&
+                                 ring_head + skip + need - meta[o].tail_snap <= uint32_t(kRingWords);
             uint32_t base = kPre;
             if (in_ring) {
                 base = (ring_head + skip) % (kRingWords ? kRingWords : 1) + 4u;
@@ -450,14 +506,25 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
 
             // a6: compact the kept words: rank r -> ring[base + r], or in place
             // -> stage[kPre + r] (every ranker's words are in registers).
+            // Partition also places the false words, in input order, after the
+            // trues: the f-th false word goes to stage[kPre + total + f], where
+            // f = (valid words before it in the tile) - (true words before it).
             uint32_t* out = (in_ring ? ring : stage) + base;
+            const uint32_t vstart = tb < p.lo ? uint32_t(p.lo - tb) : 0u;  // invalid lead words (tile 0)
 #pragma unroll
             for (int g = 0; g < kGroups; ++g) {
                 uint32_t r = wbase + ((goff >> (16 * g)) & 0xFFFFu) + ((lane_pre >> (16 * g)) & 0xFFFFu);
                 const uint32_t m = masks >> (kGroup * g);
+                const int x = kSeg * rw + 32 * kGroup * g + kGroup * lane;
 #pragma unroll
-                for (int kk = 0; kk < kGroup; ++kk)
-                    if (m >> kk & 1u) out[r++] = v[g][kk];
+                for (int kk = 0; kk < kGroup; ++kk) {
+                    if (m >> kk & 1u) {
+                        out[r++] = v[g][kk];
+                    } else if (PART) {
+                        const uint64_t e = tb + x + kk;
+                        if (e >= p.lo && e < p.hi) out[total + (uint32_t(x + kk) - vstart) - r] = v[g][kk];
+                    }
+                }
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is in the ring
@@ -511,55 +578,23 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 trace_event(p.trace, t, 5, globaltimer());
                 debug_delay(t, 3);
             }
-            // a7: chunk c covers virtual words c0 + 4c + [0, 4) = ranks 4c - ph + [0, 4)
-            // (ph = 16-byte phase of the output start), read as two aligned vectors
-            // of the ring and funnel-shifted.
+            // a7: the kept words -> [excl, excl + A) of the true output; for a
+            // partition also the false words -> [excl_false, ...) of the false output.
             const bool in_ring = meta[o].in_ring != 0;
             const int s_in = k % kInStages;
-            const uint32_t* src = (in_ring ? ring : smem + s_in * kStageWords) + meta[o].ring_base;
+            const uint32_t* buf = in_ring ? ring : smem + s_in * kStageWords;
+            const int32_t rb = int32_t(meta[o].ring_base);
             const uint32_t A = meta[o].total;
-            const uint64_t s0 = p.lo + meta[o].excl;
-            const uint64_t s1 = s0 + A;
-            const uint64_t c0 = s0 & ~3ull;
-            const uint32_t ph = uint32_t(s0 & 3);
-#ifdef DS_DEBUG_NO_STORE  // timing experiment only: no output written
-            const uint32_t nchunks = 0;
-#else
-            const uint32_t nchunks = A ? uint32_t((s1 - c0 + 3) >> 2) : 0u;
-#endif
-            // Four chunks per thread per iteration: all shared loads first, then the
-            // global stores (ILP).
-            constexpr int kU = 4;
-            for (uint32_t c0i = st; c0i < nchunks; c0i += kU * kST) {
-                uint32_t w[kU][4];
-#pragma unroll
-                for (int u = 0; u < kU; ++u) {
-                    const uint32_t c = c0i + u * kST;
-                    if (c < nchunks) {
-                        const u32x4 hi = *reinterpret_cast<const u32x4*>(src + 4 * c);
-                        const u32x4 lo = *reinterpret_cast<const u32x4*>(src + 4 * c - 4);
-                        switch (ph) {  // warp-uniform
-                        case 0: w[u][0] = hi.x; w[u][1] = hi.y; w[u][2] = hi.z; w[u][3] = hi.w; break;
-                        case 1: w[u][0] = lo.w; w[u][1] = hi.x; w[u][2] = hi.y; w[u][3] = hi.z; break;
-                        case 2: w[u][0] = lo.z; w[u][1] = lo.w; w[u][2] = hi.x; w[u][3] = hi.y; break;
-                        default: w[u][0] = lo.y; w[u][1] = lo.z; w[u][2] = lo.w; w[u][3] = hi.x; break;
-                        }
-                    }
-                }
-#pragma unroll
-                for (int u = 0; u < kU; ++u) {
-                    const uint32_t c = c0i + u * kST;
-                    if (c >= nchunks) break;
-                    const uint64_t g = c0 + 4ull * c;
-                    if (g >= s0 && g + 4 <= s1) {
-                        stg_stream_v4(p.abase + g, w[u][0], w[u][1], w[u][2], w[u][3]);
-                    } else {
-#pragma unroll
-                        for (int kk = 0; kk < 4; ++kk)
-                            if (g + kk >= s0 && g + kk < s1) stg_stream(p.abase + g + kk, w[u][kk]);
-                    }
-                }
+#ifndef DS_DEBUG_NO_STORE  // timing experiment only: no output written
+            store_segment<kST>(p.tbase, p.tlo + meta[o].excl, A, buf, rb, st);
+            if (PART) {
+                const uint64_t tb = uint64_t(t) * kT;
+                const uint64_t vs = tb > p.lo ? tb : p.lo;
+                const uint64_t ve = tb + kT < p.hi ? tb + kT : p.hi;
+                const uint64_t excl_f = (vs - p.lo) - meta[o].excl;
+                store_segment<kST>(p.fbase, p.flo + excl_f, uint32_t(ve - vs) - A, buf, rb + int32_t(A), st);
             }
+#endif
             named_bar_sync(2, kST);  // every storer is done reading the tile's ring space
             if (st == 0) {
                 trace_event(p.trace, t, 6, globaltimer());
@@ -575,10 +610,10 @@ struct LaunchCache {
     int dev = -1, sms = 0, per_sm = 0;
 };
 
-template <class Op>
+template <class Op, bool PART = false>
 cudaError_t launch_op(IrregParams p, cudaStream_t s) {
     static thread_local LaunchCache lc;
-    auto kern = irregular_kernel<Op>;
+    auto kern = irregular_kernel<Op, PART>;
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -622,19 +657,29 @@ cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s) 
     p.ntiles = uint32_t(irregular_tiles(a));
     p.value = a.value;
     p.trace = debug_trace(p.ntiles);
+    uint32_t* tptr = a.out_true ? a.out_true : a.ptr;
+    const uint64_t tmis = (reinterpret_cast<uintptr_t>(tptr) >> 2) & 3u;
+    p.tbase = tptr - tmis;
+    p.tlo = tmis;
+    if (a.out_false) {
+        const uint64_t fmis = (reinterpret_cast<uintptr_t>(a.out_false) >> 2) & 3u;
+        p.fbase = a.out_false - fmis;
+        p.flo = fmis;
+    }
     count_launch();
+    const bool part = a.out_false != nullptr;
     switch (a.op) {
     case IrregOp::Compact: return launch_op<OpCompact>(p, s);
     case IrregOp::Unique: return launch_op<OpUnique>(p, s);
     case IrregOp::Select:
         switch (a.predicate) {
-        case 0: return launch_op<OpSelect<0>>(p, s);
-        case 1: return launch_op<OpSelect<1>>(p, s);
-        case 2: return launch_op<OpSelect<2>>(p, s);
-        case 3: return launch_op<OpSelect<3>>(p, s);
-        case 4: return launch_op<OpSelect<4>>(p, s);
-        case 5: return launch_op<OpSelect<5>>(p, s);
-        case 6: return launch_op<OpSelect<6>>(p, s);
+        case 0: return part ? launch_op<OpSelect<0>, true>(p, s) : launch_op<OpSelect<0>>(p, s);
+        case 1: return part ? launch_op<OpSelect<1>, true>(p, s) : launch_op<OpSelect<1>>(p, s);
+        case 2: return part ? launch_op<OpSelect<2>, true>(p, s) : launch_op<OpSelect<2>>(p, s);
+        case 3: return part ? launch_op<OpSelect<3>, true>(p, s) : launch_op<OpSelect<3>>(p, s);
+        case 4: return part ? launch_op<OpSelect<4>, true>(p, s) : launch_op<OpSelect<4>>(p, s);
+        case 5: return part ? launch_op<OpSelect<5>, true>(p, s) : launch_op<OpSelect<5>>(p, s);
+        case 6: return part ? launch_op<OpSelect<6>, true>(p, s) : launch_op<OpSelect<6>>(p, s);
         default: return cudaErrorInvalidValue;
         }
     }

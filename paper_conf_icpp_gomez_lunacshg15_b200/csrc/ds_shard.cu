@@ -32,7 +32,34 @@ __global__ void shard_offsets_kernel(const uint64_t* counts, uint32_t world, uin
     }
 }
 
+// Partition's second step ("move the false elements from the
+// auxiliary buffer to the tail of Array, once the true elements have been
+// shifted"): dst_base[*d_offset + j] = src[j] for j < n_total - *d_offset.
+// Grid-stride, one word per thread per iteration (coalesced on both sides).
+__global__ void tail_copy_kernel(uint32_t* dst_base, const uint64_t* d_offset, const uint32_t* src,
+                                 uint64_t n_total) {
+    const uint64_t off = *d_offset;
+    const uint64_t cnt = n_total - off;
+    uint32_t* dst = dst_base + off;
+    for (uint64_t j = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; j < cnt;
+         j += uint64_t(gridDim.x) * blockDim.x)
+        dst[j] = src[j];
+}
+
 }  // namespace
+
+cudaError_t launch_tail_copy(uint32_t* dst_base, const uint64_t* d_offset, const uint32_t* src,
+                             const uint64_t* /*d_count_false*/, size_t n_total, cudaStream_t s) {
+    count_launch();
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    uint64_t blocks = (n_total + 255) / 256;
+    if (blocks > uint64_t(sms) * 8) blocks = uint64_t(sms) * 8;
+    if (blocks == 0) blocks = 1;
+    tail_copy_kernel<<<uint32_t(blocks), 256, 0, s>>>(dst_base, d_offset, src, n_total);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_halo_entry(const uint32_t* ptr, size_t n, uint64_t* d_entry, cudaStream_t s) {
     count_launch();

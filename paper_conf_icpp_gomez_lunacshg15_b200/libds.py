@@ -33,6 +33,10 @@ SIGNATURES = {
     "ds_compact_ex": (_i, [_vp, _sz, _u32, _vp, _vp]),
     "ds_select_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp]),
     "ds_unique_ex": (_i, [_vp, _sz, _vp, _sz, _vp, _vp]),
+    "ds_partition": (_i, [_vp, _sz, _i, _vp, _psz]),
+    "ds_partition_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp, _vp]),
+    "ds_select_copy_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp, _vp]),
+    "ds_partition_copy_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp, _vp, _vp]),
     "ds_halo_entry": (_i, [_vp, _sz, _vp, _vp]),
     "ds_shard_offsets": (_i, [_vp, _sz, _sz, _vp, _vp]),
     "ds_status_string": (ctypes.c_char_p, [_i]),
@@ -157,6 +161,30 @@ def ds_select_ex(ptr, n: int, predicate_id: int, param: int = 0, d_out_n=None, s
 def ds_unique_ex(ptr, n: int, d_halo=None, halo_len: int = 0, d_out_n=None, stream=None) -> None:
     _check(_lib.ds_unique_ex(_addr(ptr), n, _addr(d_halo), halo_len, _addr(d_out_n),
                              _stream(stream)), "ds_unique_ex")
+
+
+# ------------------------------------------------- partition / out-of-place
+def ds_partition(ptr, n: int, predicate_id: int, aux) -> int:
+    out = ctypes.c_size_t(0)
+    _check(_lib.ds_partition(_addr(ptr), n, predicate_id, _addr(aux), ctypes.byref(out)), "ds_partition")
+    return out.value
+
+
+def ds_partition_ex(ptr, n: int, predicate_id: int, param: int, aux, d_out_n_true, stream=None) -> None:
+    _check(_lib.ds_partition_ex(_addr(ptr), n, predicate_id, param & 0xFFFFFFFF, _addr(aux),
+                                _addr(d_out_n_true), _stream(stream)), "ds_partition_ex")
+
+
+def ds_select_copy_ex(src, n: int, predicate_id: int, param: int, out, d_out_n=None, stream=None) -> None:
+    _check(_lib.ds_select_copy_ex(_addr(src), n, predicate_id, param & 0xFFFFFFFF, _addr(out),
+                                  _addr(d_out_n), _stream(stream)), "ds_select_copy_ex")
+
+
+def ds_partition_copy_ex(src, n: int, predicate_id: int, param: int, out_true, out_false,
+                         d_out_n_true=None, stream=None) -> None:
+    _check(_lib.ds_partition_copy_ex(_addr(src), n, predicate_id, param & 0xFFFFFFFF, _addr(out_true),
+                                     _addr(out_false), _addr(d_out_n_true), _stream(stream)),
+           "ds_partition_copy_ex")
 
 
 # ------------------------------------------------------------------ sharding

@@ -125,3 +125,12 @@ def test_binding_rejects_host_tensors():
     t = torch.zeros(8, dtype=torch.int32)
     with pytest.raises(ValueError):
         libds.ds_compact(t, 8, 0)
+
+
+def test_partition_and_copy_validation():
+    assert st("ds_partition", FAKE, 10, 0, None, out_sz()) == INV        # no aux
+    assert st("ds_partition", FAKE, 10, 9, FAKE, out_sz()) == INV        # bad predicate
+    assert st("ds_partition_ex", FAKE, 10, 0, 0, FAKE, None, None) == INV  # count required
+    assert st("ds_select_copy_ex", FAKE, 10, 0, 0, None, None, None) == INV  # no out
+    assert st("ds_select_copy_ex", FAKE, 10, 0, 0, BAD, None, None) == INV   # misaligned out
+    assert st("ds_partition_copy_ex", FAKE, 10, 0, 0, FAKE, None, None, None) == INV

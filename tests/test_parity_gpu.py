@@ -298,3 +298,72 @@ def test_pad_repeat_race_hunt():
         work.copy_(src)
         libds.ds_pad_ex(work, R, C, NC, 4, None, None)
         assert torch.equal(work, want), rep
+
+
+# ------------------------------------------------- partition / out-of-place
+@pytest.mark.parametrize("n", [1, 5, T - 1, 2 * T + 1, 3 * T + 7, 65537, 1_000_003])
+@pytest.mark.parametrize("mis", [0, 3])
+def test_partition_in_place(n, mis):
+    """Stable partition through the caller's aux buffer."""
+    for k, f in enumerate([0.0, 0.3, 0.5, 1.0]):
+        a = _u32(dsgen.select_input(n, 400 + k + n))
+        t = dsgen.select_threshold(f) & 0xFFFFFFFF
+        buf = DevBuf(a, mis)
+        exp = buf.host_region()
+        m_exp = oracle.partition(exp, oracle.PRED_I32_GT, t)
+        aux = DevBuf(np.zeros(n, dtype=np.uint32), (mis + 1) % 4)
+        d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+        libds.ds_partition_ex(buf.ptr, n, libds.DS_PRED_I32_GT, t, aux.ptr, d_n, None)
+        torch.cuda.synchronize()
+        assert int(d_n.item()) == m_exp, (n, f)
+        buf.assert_equals(exp, f"partition n={n} f={f}")
+        aux_got = aux.fetch()
+        assert np.array_equal(aux_got[:aux.pre], aux.expected_full[:aux.pre])          # canaries
+        assert np.array_equal(aux_got[aux.pre + n:], aux.expected_full[aux.pre + n:])
+
+
+def test_partition_blocking_even_odd():
+    """Fig. 18 style: evens (true) before odds, both stable; blocking form."""
+    a = _u32(dsgen.random_words(300_007, 8))
+    buf = DevBuf(a, 1)
+    exp = buf.host_region()
+    m_exp = oracle.partition(exp, oracle.PRED_I32_EVEN)
+    aux = torch.empty(a.size, dtype=torch.int32, device="cuda")
+    assert libds.ds_partition(buf.ptr, a.size, libds.DS_PRED_I32_EVEN, aux) == m_exp
+    buf.assert_equals(exp, "partition even")
+
+
+@pytest.mark.parametrize("n", [3, T + 1, 250_001])
+@pytest.mark.parametrize("mis_in,mis_out", [(0, 0), (1, 2), (3, 1)])
+def test_select_copy_out_of_place(n, mis_in, mis_out):
+    a = _u32(dsgen.random_words(n, 500 + n))
+    src = DevBuf(a, mis_in)
+    out = DevBuf(np.full(n, 0x12345678, dtype=np.uint32), mis_out)
+    exp_out = out.host_region()
+    kept = oracle.select_copy(a, oracle.PRED_F32_GT, 0x3F000000)
+    exp_out[:kept.size] = kept
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    libds.ds_select_copy_ex(src.ptr, n, libds.DS_PRED_F32_GT, 0x3F000000, out.ptr, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == kept.size
+    out.assert_equals(exp_out, "select_copy out")
+    src.assert_equals(a, "select_copy input unchanged")
+
+
+@pytest.mark.parametrize("n", [7, 2 * T + 3, 400_009])
+def test_partition_copy_out_of_place(n):
+    a = _u32(dsgen.random_words(n, 600 + n))
+    src = DevBuf(a, 2)
+    ot = DevBuf(np.zeros(n, dtype=np.uint32), 1)
+    of = DevBuf(np.zeros(n, dtype=np.uint32), 3)
+    keep = (a & 1) == 1
+    et, ef = ot.host_region(), of.host_region()
+    et[:keep.sum()] = a[keep]
+    ef[:(~keep).sum()] = a[~keep]
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    libds.ds_partition_copy_ex(src.ptr, n, libds.DS_PRED_I32_ODD, 0, ot.ptr, of.ptr, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == int(keep.sum())
+    ot.assert_equals(et, "trues")
+    of.assert_equals(ef, "falses")
+    src.assert_equals(a, "input unchanged")
