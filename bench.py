@@ -180,6 +180,23 @@ def bench_rows(peak, flush):
         irregular("unique", f"C3 256M int32 runs f={f:.1f}", src,
                   lambda w: libds.ds_unique_ex(w, n, None, 0, d_n, None), reps=3)
         del src
+    # Partition (in place through an aux buffer) and out-of-place
+    # select (Copy_if) on 256M int32 at 50 %
+    n = 1 << 28
+    src = dsgen.select_input(n, dsgen.seed_for(5), device="cuda")
+    t = dsgen.select_threshold(0.5) & 0xFFFFFFFF
+    aux = torch.empty_like(src)
+    work = torch.empty_like(src)
+    ms = timed(lambda: libds.ds_partition_ex(work, n, libds.DS_PRED_I32_GT, t, aux, d_n, None), s,
+               restore=lambda: work.copy_(src), flush=flush, reps=3)
+    m = int(d_n.item())
+    row("partition", "256M int32 x>t f=0.5 (in place, aux)", ms, 4 * (2 * n + 2 * (n - m)),
+        {"n": n, "out_n": m, "bytes": "read n + write n_true in place + write/read/write n_false via aux"})
+    ms = timed(lambda: libds.ds_select_copy_ex(src, n, libds.DS_PRED_I32_GT, t, work, d_n, None), s,
+               flush=flush, reps=3)
+    m = int(d_n.item())
+    row("select_copy", "256M int32 x>t f=0.5 (out of place)", ms, 4 * (n + m), {"n": n, "out_n": m})
+    del src, aux, work
     # C4: 1G float32 compaction at 10 / 50 / 90 %
     n = 1 << 30
     for f in (0.1, 0.5, 0.9):
