@@ -97,6 +97,19 @@ ds_status ds_pad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols,
 ds_status ds_unpad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols,
                       size_t elem_bytes, ds_stream_t stream);
 
+/* ds_slide -- the one-group regular DS: "groups of consecutive input array
+ * elements are shifted by a constant amount of memory positions",
+ * here a single group moved backward by `shift` elements in place:
+ * elements [shift, n) of ptr move to [0, n - shift), order kept; elements
+ * [n - shift, n) keep their old bytes (R5).  Same tiles, LOADED windows and
+ * kernel as ds_unpad (Algorithm 1).  Requires shift <= n;
+ * elem_bytes in {4, 8, 16}.  Used by the multi-GPU rebalance (DESIGN.md
+ * section 5) to close a shard's gap after its head was sent to a lower
+ * rank.                                                                  */
+ds_status ds_slide(void* ptr, size_t n, size_t shift, size_t elem_bytes);
+ds_status ds_slide_ex(void* ptr, size_t n, size_t shift, size_t elem_bytes,
+                      ds_stream_t stream);
+
 /* ---------------------------------------------------------------------
  * Irregular DS (Algorithm 2)
  * ------------------------------------------------------------------- */

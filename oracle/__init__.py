@@ -63,6 +63,8 @@ def lib():
         L.oracle_pad.restype = i32
         L.oracle_unpad.argtypes = [vp, sz, sz, sz, sz]
         L.oracle_unpad.restype = i32
+        L.oracle_slide.argtypes = [vp, sz, sz, sz]
+        L.oracle_slide.restype = i32
         _lib = L
     return _lib
 
@@ -156,3 +158,13 @@ def unpad(buf: np.ndarray, rows: int, cols: int, new_cols: int, elem_bytes: int)
     rc = lib().oracle_unpad(_ptr(buf), rows, cols, new_cols, elem_bytes)
     if rc != 0:
         raise ValueError("oracle_unpad: new_cols > cols or elem_bytes == 0")
+
+
+def slide(buf: np.ndarray, n: int, shift: int, elem_bytes: int) -> None:
+    """In place on the raw bytes of ``buf``: elements [shift, n) -> [0, n - shift)."""
+    buf = _bytes_view(buf)
+    if n * elem_bytes > buf.nbytes:
+        raise ValueError("buffer too small")
+    rc = lib().oracle_slide(_ptr(buf), n, shift, elem_bytes)
+    if rc != 0:
+        raise ValueError("oracle_slide: shift > n or elem_bytes == 0")

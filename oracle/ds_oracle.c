@@ -128,3 +128,14 @@ int oracle_unpad(uint8_t* b, size_t rows, size_t cols, size_t new_cols,
     }
     return 0;
 }
+
+/* every element of the single group moves by the same constant; the
+ * move is backward, so go from the first element on (no element is
+ * overwritten before it was moved).                                      */
+int oracle_slide(uint8_t* b, size_t n, size_t shift, size_t elem_bytes) {
+    if (shift > n || elem_bytes == 0) return -1;
+    for (size_t i = shift; i < n; ++i)
+        for (size_t k = 0; k < elem_bytes; ++k)
+            b[(i - shift) * elem_bytes + k] = b[i * elem_bytes + k];
+    return 0;
+}

@@ -100,6 +100,13 @@ int oracle_pad(uint8_t* b, size_t rows, size_t cols, size_t new_cols,
 int oracle_unpad(uint8_t* b, size_t rows, size_t cols, size_t new_cols,
                  size_t elem_bytes);
 
+/* Slide, the one-group regular DS ("groups of consecutive input
+ * array elements are shifted by a constant amount of memory positions"):
+ * elements [shift, n) (elem_bytes each) move backward by `shift` to
+ * [0, n - shift), in input order; elements [n - shift, n) keep their bytes
+ * (R5).  Returns 0, or -1 if shift > n or elem_bytes == 0.               */
+int oracle_slide(uint8_t* b, size_t n, size_t shift, size_t elem_bytes);
+
 #ifdef __cplusplus
 }
 #endif

@@ -207,6 +207,42 @@ ds_status ds_unpad(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t 
     return st == DS_SUCCESS ? sync_default() : st;
 }
 
+ds_status ds_slide_ex(void* ptr, size_t n, size_t shift, size_t elem_bytes, ds_stream_t stream) {
+    if (elem_bytes == 1 || elem_bytes == 2) return DS_ERROR_UNSUPPORTED;
+    if (elem_bytes != 4 && elem_bytes != 8 && elem_bytes != 16) return DS_ERROR_INVALID_VALUE;
+    if (shift > n) return DS_ERROR_INVALID_VALUE;
+    size_t bytes = 0;
+    if (__builtin_mul_overflow(n, elem_bytes, &bytes)) return DS_ERROR_INVALID_VALUE;
+    if (n > 0 && ptr == nullptr) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(ptr, 4)) return DS_ERROR_INVALID_VALUE;
+    if (bytes / 4 > kMaxMatrixWords) return DS_ERROR_UNSUPPORTED;
+    if (shift == 0 || shift == n) return DS_SUCCESS;  // nothing moves
+    // A regular DS with one group: unpad geometry with equal row lengths and
+    // a source offset (rows of kSlideRow words; any length works).
+    constexpr uint64_t kSlideRow = 1ull << 20;
+    const uint64_t w = elem_bytes / 4;
+    ds::RegArgs a{};
+    a.ptr = static_cast<uint32_t*>(ptr);
+    a.out_words_w = uint64_t(n - shift) * w;
+    a.src0_w = uint64_t(shift) * w;
+    a.cols_w = a.new_cols_w = kSlideRow;
+    a.rows = (a.out_words_w + kSlideRow - 1) / kSlideRow;
+    a.words_per_elem = uint32_t(w);
+    a.pad = false;
+    std::lock_guard<std::mutex> lock(g_mu);
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    ds::Workspace* ws = nullptr;
+    ds_status st = get_workspace(ds::regular_tiles(a), s, &ws);
+    if (st != DS_SUCCESS) return st;
+    cudaError_t e = ds::launch_regular(a, *ws, s);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "regular kernel launch");
+}
+
+ds_status ds_slide(void* ptr, size_t n, size_t shift, size_t elem_bytes) {
+    ds_status st = ds_slide_ex(ptr, n, shift, elem_bytes, nullptr);
+    return st == DS_SUCCESS ? sync_default() : st;
+}
+
 ds_status ds_compact_ex(void* ptr, size_t n, uint32_t remove_value, uint64_t* d_out_n,
                         ds_stream_t stream) {
     ds_status st = check_irregular(ptr, n, d_out_n);

@@ -42,6 +42,8 @@ struct RegArgs {
     uint32_t words_per_elem;
     uint32_t fill[4];
     bool pad;             // true: pad (expand, descending), false: unpad
+    uint64_t src0_w = 0;       // slide: source word offset (unpad geometry with Cw == NCw)
+    uint64_t out_words_w = 0;  // slide: output words (0: rows * new_cols_w)
 };
 
 // Tiles a launch of each kernel family needs (for workspace sizing).

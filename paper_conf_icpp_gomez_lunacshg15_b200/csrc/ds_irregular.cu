@@ -116,6 +116,10 @@ constexpr int kRingWords = DS_IRR_RING_WORDS; // compacted tiles awaiting their 
 constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
 constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
 constexpr int kStoreWarps = 5;
+#ifndef DS_IRR_BULK_STORE
+#define DS_IRR_BULK_STORE 1
+#endif
+constexpr bool kBulkStore = DS_IRR_BULK_STORE;  // a7 through TMA bulk stores (else 128-bit STG)
 constexpr int kST = 32 * kStoreWarps;
 constexpr int kWarpResolver0 = kRankWarps;
 constexpr int kWarpStorer0 = kRankWarps + kResolvers;
@@ -201,11 +205,18 @@ constexpr int kRefreshRows = DS_IRR_REFRESH;        // AGG rows re-read while po
 constexpr uint32_t kPollMinNs = DS_IRR_POLL_MIN;   // first back-off
 constexpr uint32_t kPollMaxNs = DS_IRR_POLL_MAX;   // back-off cap
 
-__device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status, uint32_t tile,
+#ifndef DS_IRR_HELP
+#define DS_IRR_HELP 0
+#endif
+constexpr bool kHelp = DS_IRR_HELP;  // publish INCL for the nearest 32 AGG predecessors
+
+__device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint32_t tile,
                                              uint32_t epoch, int lane, uint64_t* trace) {
     uint64_t excl = 0;
     uint32_t rounds = 0, polls = 0;
     int64_t base = int64_t(tile) - 1;
+    uint64_t s0 = 0;     // the nearest 32 predecessors' statuses as the first round left them
+    uint32_t L0 = 32u;   // lanes of that row the walk needed (up to the nearest INCL)
     while (true) {
         uint64_t s[kLB];
         uint32_t okm = 0;  // bit m: slot m holds a current status
@@ -259,11 +270,33 @@ __device__ __forceinline__ uint64_t lookback(const uint64_t* __restrict__ status
             if (uint32_t(m) == M && uint32_t(lane) == L) inc = status_count(s[m]);
         }
         excl += uint64_t(__reduce_add_sync(kFull, agg));
+        if (rounds == 1) {
+            s0 = s[0];
+            L0 = M == 0 ? L : 32u;
+        }
         if (M < kLB) {
             excl += __shfl_sync(kFull, inc, L);
             break;
         }
         base -= 32 * kLB;
+    }
+    if (kHelp) {
+        // The walk fixed the inclusive prefix of every tile it summed: for the
+        // nearest predecessors t-1-l (l < L0, all AGG), incl = excl - (counts of
+        // t-1 .. t-l).  Publishing them lets later look-backs stop sooner.  A
+        // racing writer (the tile's own resolver, another helper) stores the
+        // same word.
+        const uint32_t c0 = uint32_t(lane) < L0 ? uint32_t(status_count(s0)) : 0u;
+        uint32_t pre = c0;
+#pragma unroll
+        for (int sh = 1; sh < 32; sh <<= 1) {
+            const uint32_t y = __shfl_up_sync(kFull, pre, sh);
+            if (lane >= sh) pre += y;
+        }
+        pre -= c0;  // exclusive: counts of the lanes nearer than this one
+        const int64_t idx = int64_t(tile) - 1 - lane;
+        if (uint32_t(lane) < L0 && idx >= 0 && status_state(s0) == kStateAgg)
+            publish_status(status_ptr(status, idx), make_status(kStateIncl, epoch, excl - pre));
     }
     if (lane == 0) {
         trace_event(trace, tile, 8, rounds);
@@ -323,6 +356,42 @@ __device__ __forceinline__ void store_segment(uint32_t* base, uint64_t d0, uint3
                     if (g + kk >= d0 && g + kk < d1) stg_stream(base + g + kk, w[u][kk]);
             }
         }
+    }
+}
+
+// a7 helper: move the cnt words seg[0, cnt) to seg[ph, ph + cnt) in shared
+// memory (ph = 1..3; seg 16-byte aligned with >= 4 readable words before it
+// and >= 4 writable words after the segment).  Destination chunk c (words
+// [4c, 4c+4)) takes source words [4c-ph, 4c+4-ph): two aligned vector loads.
+// Writing chunk c destroys sources of chunk c+1 only, so the chunks go in
+// descending rounds, each reading everything before writing.
+template <int kSTT>
+__device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph, int st) {
+    constexpr int kU = 4;
+    const int32_t nchunks = int32_t((cnt + ph + 3) >> 2);
+    for (int32_t hi = nchunks; hi > 0; hi -= kU * kSTT) {
+        const int32_t lo = hi - kU * kSTT;
+        u32x4 w[kU];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int32_t c = lo + u * kSTT + st;
+            if (c >= 0 && c < hi) {
+                const u32x4 a = *reinterpret_cast<const u32x4*>(seg + 4 * c - 4);
+                const u32x4 b = *reinterpret_cast<const u32x4*>(seg + 4 * c);
+                switch (ph) {  // uniform
+                case 1: w[u] = u32x4{a.w, b.x, b.y, b.z}; break;
+                case 2: w[u] = u32x4{a.z, a.w, b.x, b.y}; break;
+                default: w[u] = u32x4{a.y, a.z, a.w, b.x}; break;
+                }
+            }
+        }
+        named_bar_sync(2, kSTT);
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const int32_t c = lo + u * kSTT + st;
+            if (c >= 0 && c < hi) *reinterpret_cast<u32x4*>(seg + 4 * c) = w[u];
+        }
+        named_bar_sync(2, kSTT);
     }
 }
 
@@ -526,6 +595,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                     }
                 }
             }
+            fence_proxy_async_smem();  // the compacted words may leave through a bulk store
             __syncwarp();
             if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is in the ring
         }
@@ -568,7 +638,20 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         }
     } else {
         // ------------------------------------------------ storer warps
+        // a7.  Kept words go out through one TMA bulk store per tile (the
+        // aligned interior) plus <= 6 scalar head/tail words.  The stage is
+        // first re-phased in shared memory so that its words sit at the same
+        // 16-byte phase as their destination.  A tile's stage is released
+        // kStoreLag tiles later, once the bulk engine has finished reading it.
+        // Partition (two destinations) keeps the register path (store_segment).
         const int st = tid - 32 * kWarpStorer0;
+        int pend_s = -1, pend_o = -1;  // the tile whose release is pending (lag 1)
+        uint32_t pend_ring = 0, pend_in_ring = 0;
+        auto release = [&](int s_in, int o, uint32_t in_ring, uint32_t ring_end) {
+            if (in_ring) s_ring_tail = ring_end;
+            else mbar_arrive(&bar_free[s_in]);  // the in-place tile's input stage is free
+            mbar_arrive(&bar_stored[o]);
+        };
         for (uint32_t k = 0;; ++k) {
             const int o = k % kSlots;
             mbar_wait(&bar_resolved[o], (k / kSlots) & 1);
@@ -580,28 +663,71 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             }
             // a7: the kept words -> [excl, excl + A) of the true output; for a
             // partition also the false words -> [excl_false, ...) of the false output.
-            const bool in_ring = meta[o].in_ring != 0;
+            const uint32_t in_ring = meta[o].in_ring;
             const int s_in = k % kInStages;
-            const uint32_t* buf = in_ring ? ring : smem + s_in * kStageWords;
+            uint32_t* buf = in_ring ? ring : smem + s_in * kStageWords;
             const int32_t rb = int32_t(meta[o].ring_base);
             const uint32_t A = meta[o].total;
+            const uint64_t tb0 = uint64_t(t) * kT;
+            const uint64_t vs0 = tb0 > p.lo ? tb0 : p.lo;
+            const uint64_t ve0 = tb0 + kT < p.hi ? tb0 + kT : p.hi;
 #ifndef DS_DEBUG_NO_STORE  // timing experiment only: no output written
-            store_segment<kST>(p.tbase, p.tlo + meta[o].excl, A, buf, rb, st);
-            if (PART) {
-                const uint64_t tb = uint64_t(t) * kT;
-                const uint64_t vs = tb > p.lo ? tb : p.lo;
-                const uint64_t ve = tb + kT < p.hi ? tb + kT : p.hi;
-                const uint64_t excl_f = (vs - p.lo) - meta[o].excl;
-                store_segment<kST>(p.fbase, p.flo + excl_f, uint32_t(ve - vs) - A, buf, rb + int32_t(A), st);
+            if (PART || !kBulkStore) {
+                if (!PART && p.tbase == p.abase && meta[o].excl == vs0 - p.lo && A == ve0 - vs0) {
+                    // identity tile: nothing to store
+                } else {
+                    store_segment<kST>(p.tbase, p.tlo + meta[o].excl, A, buf, rb, st);
+                }
+                if (PART) {
+                    const uint64_t excl_f = (vs0 - p.lo) - meta[o].excl;
+                    store_segment<kST>(p.fbase, p.flo + excl_f, uint32_t(ve0 - vs0) - A, buf, rb + int32_t(A), st);
+                }
+            } else {
+                // Identity tile (in place, nothing removed in or before it): every
+                // kept word would be written onto itself, so the stores are skipped.
+                const bool identity = p.tbase == p.abase && meta[o].excl == vs0 - p.lo && A == ve0 - vs0;
+                if (!identity && A > 0) {
+                    const uint64_t d0 = p.tlo + meta[o].excl, d1 = d0 + A;
+                    const uint32_t ph = uint32_t(d0) & 3u;
+                    uint32_t* seg = buf + rb;  // 16-byte aligned (rb % 4 == 0)
+                    if (ph) rephase<kST>(seg, A, ph, st);  // word r -> seg[ph + r]
+                    const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
+                    if (g1 > g0) {
+                        fence_proxy_async_smem();  // re-phased words -> visible to the bulk engine
+                        named_bar_sync(2, kST);
+                        if (st == 0)
+                            bulk_s2g(p.tbase + g0, seg + ph + uint32_t(g0 - d0), uint32_t(g1 - g0) * 4u);
+                        // head [d0, g0) and tail [g1, d1): at most 3 words each
+                        if (st < 3 && d0 + st < g0) stg_stream(p.tbase + d0 + st, seg[ph + st]);
+                        if (st >= 3 && st < 6 && g1 + (st - 3) < d1)
+                            stg_stream(p.tbase + g1 + (st - 3), seg[ph + uint32_t(g1 - d0) + (st - 3)]);
+                    } else {
+                        named_bar_sync(2, kST);
+                        if (uint32_t(st) < A) stg_stream(p.tbase + d0 + st, seg[ph + st]);  // A < 8
+                    }
+                }
             }
 #endif
-            named_bar_sync(2, kST);  // every storer is done reading the tile's ring space
+            named_bar_sync(2, kST);  // every storer is done reading the tile's stage
             if (st == 0) {
                 trace_event(p.trace, t, 6, globaltimer());
-                if (in_ring) s_ring_tail = meta[o].ring_end;
-                else mbar_arrive(&bar_free[s_in]);  // the in-place tile's input stage is free
-                mbar_arrive(&bar_stored[o]);
+                bulk_commit();  // (possibly empty) group of this tile
+                if (PART || !kBulkStore) {
+                    release(s_in, o, in_ring, meta[o].ring_end);
+                } else {
+                    bulk_wait_read<1>();  // the previous tile's stage has been read
+                    if (pend_o >= 0) release(pend_s, pend_o, pend_in_ring, pend_ring);
+                    pend_s = s_in;
+                    pend_o = o;
+                    pend_in_ring = in_ring;
+                    pend_ring = meta[o].ring_end;
+                }
             }
+        }
+        if (st == 0) {
+            bulk_wait_read<0>();
+            if (pend_o >= 0) release(pend_s, pend_o, pend_in_ring, pend_ring);
+            bulk_wait_all();  // the bulk stores are complete before the CTA exits
         }
     }
 }

@@ -40,7 +40,8 @@ constexpr int64_t kNoTile = -1;
 struct RegParams {
     uint32_t* abase;  // 16-byte-aligned base; virtual word 0
     uint64_t mis;     // ptr - abase in words
-    uint64_t out_words, in_words;
+    uint64_t out_words, in_words;  // in_words: physical end of the sources (src0 + rows*Cw)
+    int64_t src0;     // slide: source of output word q is src0 + q (unpad geometry, Cw == NCw)
     uint32_t Cw, NCw;
     FastDiv div_nc;
     FastDiv64 div_nc64, div_c64;
@@ -86,8 +87,8 @@ __device__ void tile_geometry(const RegParams& p, int64_t k, TileGeom& g) {
         slo = g.col0 < Cw ? g.row0 * Cw + g.col0 : (g.row0 + 1) * Cw;
         shi = col1 < Cw ? row1 * Cw + col1 : row1 * Cw + Cw - 1;
     } else {
-        slo = g.row0 * Cw + g.col0;
-        shi = row1 * Cw + col1;
+        slo = p.src0 + g.row0 * Cw + g.col0;
+        shi = p.src0 + row1 * Cw + col1;
     }
     g.slo = slo;
     g.span = shi >= slo ? shi - slo + 1 : 0;
@@ -95,11 +96,12 @@ __device__ void tile_geometry(const RegParams& p, int64_t k, TileGeom& g) {
     const int64_t se = (slo + mis + g.span + 3) & ~int64_t(3);  // may pass the end by <= 3 words
     g.fast = (se - g.sb) <= STAGE;
     g.bytes = g.span > 0 && g.fast ? uint32_t(se - g.sb) * 4u : 0u;
-    g.base_rel = int32_t(g.row0 * Cw - slo);
+    g.base_rel = int32_t(p.src0 + g.row0 * Cw - slo);
 
-    // Sources physically inside this tile's output range: input words [P0, P1).
-    const int64_t P0 = g.q0;
-    const int64_t P1 = g.q1 < int64_t(p.in_words) ? g.q1 : int64_t(p.in_words);
+    // Sources physically inside this tile's output range: input words [P0, P1)
+    // (source indices; a slide's sources start at physical word src0).
+    const int64_t P0 = g.q0 - p.src0 > 0 ? g.q0 - p.src0 : 0;
+    const int64_t P1 = (g.q1 < int64_t(p.in_words) ? g.q1 : int64_t(p.in_words)) - p.src0;
     g.win_lo = 1;
     g.win_hi = 0;
     if (P0 < P1) {
@@ -184,7 +186,7 @@ __device__ void gather_slow(const RegParams& p, const TileGeom& g, uint32_t* sta
                 const uint32_t dr = fastdiv(t, p.div_nc);
                 const uint32_t col = t - dr * p.NCw;
                 if (PAD && col >= p.Cw) val[u] = fill_word(p, col);
-                else val[u] = ldg_stream(p.abase + (g.row0 + dr) * int64_t(p.Cw) + col + mis);
+                else val[u] = ldg_stream(p.abase + p.src0 + (g.row0 + dr) * int64_t(p.Cw) + col + mis);
             }
         }
 #pragma unroll
@@ -413,7 +415,7 @@ cudaError_t launch_dir(RegParams p, cudaStream_t s) {
 
 size_t regular_tiles(const RegArgs& a) {
     const uint64_t mis = (reinterpret_cast<uintptr_t>(a.ptr) >> 2) & 3u;
-    const uint64_t out_words = a.rows * a.new_cols_w;
+    const uint64_t out_words = a.out_words_w ? a.out_words_w : a.rows * a.new_cols_w;
     return size_t((out_words + mis + kT - 1) / kT);
 }
 
@@ -422,8 +424,9 @@ cudaError_t launch_regular(const RegArgs& a, Workspace& ws, cudaStream_t s) {
     const uint64_t mis = (reinterpret_cast<uintptr_t>(a.ptr) >> 2) & 3u;
     p.abase = a.ptr - mis;
     p.mis = mis;
-    p.out_words = a.rows * a.new_cols_w;
-    p.in_words = a.rows * a.cols_w;
+    p.out_words = a.out_words_w ? a.out_words_w : a.rows * a.new_cols_w;
+    p.src0 = int64_t(a.src0_w);
+    p.in_words = a.out_words_w ? a.src0_w + a.out_words_w : a.rows * a.cols_w;
     p.Cw = uint32_t(a.cols_w);
     p.NCw = uint32_t(a.new_cols_w);
     p.div_nc = make_fastdiv(p.NCw);

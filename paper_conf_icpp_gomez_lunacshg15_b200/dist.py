@@ -13,12 +13,25 @@ Unique needs one more 8-byte all-gather *before* the slide: each shard's
 (non-empty, last word) "halo" entry, so that a shard's first word is
 compared with the last word of the nearest non-empty earlier shard (R18).
 
+Optional rebalance: ``rebalance`` turns the ragged
+layout into the contiguous one -- global output g lands where input word g
+lived, i.e. exactly what one in-place DS of the whole distributed array
+would leave (rank r holds outputs [B_r, B_{r+1}) clipped to out_n, B_r the
+shard starts).  Every output moves to a lower or equal global position
+(out(p) <= p), so data only flows to lower ranks: each rank sends its
+first min(c_r, d_r) outputs (d_r = B_r - off_r >= 0) to the ranks below,
+closes the gap with one in-place regular DS (ds_slide by d_r), then
+receives from higher ranks.  A rank may receive only after its own send
+and slide, so the ranks go in "waves" (wave = 1 + the largest wave of the
+ranks it sends to); each wave is one batch of NCCL send/recv over NVLink.
+
 The device steps are delegated to a ``local`` object; the default,
 ``LibdsLocal``, calls the libds C ABI on CUDA tensors.  Tests substitute a
 CPU stand-in to exercise the orchestration and the collectives with gloo.
 """
 from __future__ import annotations
 
+import bisect
 from dataclasses import dataclass
 
 import torch
@@ -59,6 +72,65 @@ class LibdsLocal:
     def offsets(self, d_counts, world, rank, d_result, stream=None):
         self.libds.ds_shard_offsets(d_counts, world, rank, d_result, stream)
 
+    def slide(self, shard, n, shift, stream=None):
+        self.libds.ds_slide_ex(shard if n else None, n, shift, 4, stream)
+
+
+@dataclass(frozen=True)
+class Piece:
+    """count words of rank src's local [src_lo, ...) -> rank dst's local [dst_lo, ...)."""
+    src: int
+    src_lo: int
+    dst: int
+    dst_lo: int
+    count: int
+
+
+@dataclass
+class RebalancePlan:
+    pieces: list          # every transfer between ranks
+    shift: list           # per rank: ds_slide shift (min(c_r, d_r)); 0 = no slide
+    kept: list            # per rank: words kept locally (c_r - shift)
+    wave: list            # per rank: the wave in which it sends and slides
+    final: list           # per rank: words holding outputs after the rebalance
+    total: int
+
+    @property
+    def waves(self) -> int:
+        return max(self.wave) + 1 if self.wave else 0
+
+
+def rebalance_plan(counts: list[int], sizes: list[int]) -> RebalancePlan:
+    """Host-side schedule of the rebalance from every shard's kept count and
+    capacity (pure function of the all-gathered counts; the same on every rank)."""
+    G = len(counts)
+    assert len(sizes) == G and all(0 <= c <= s for c, s in zip(counts, sizes))
+    B = [0] * (G + 1)
+    off = [0] * (G + 1)
+    for r in range(G):
+        B[r + 1] = B[r] + sizes[r]
+        off[r + 1] = off[r] + counts[r]
+    total = off[G]
+    pieces, shift, kept = [], [], []
+    for r in range(G):
+        d = B[r] - off[r]                      # >= 0: off_r <= B_r
+        assert d >= 0
+        down = min(counts[r], d)
+        shift.append(down)
+        kept.append(counts[r] - down)
+        g, end = off[r], off[r] + down        # global range going below rank r
+        while g < end:
+            q = bisect.bisect_right(B, g) - 1     # B[q] <= g < B[q+1] (skips empty shards)
+            n = min(end, B[q + 1]) - g
+            pieces.append(Piece(r, g - off[r], q, g - B[q], n))
+            g += n
+    wave = [0] * G
+    for r in range(G):                         # destinations are lower ranks: ascending order works
+        dests = [p.dst for p in pieces if p.src == r]
+        wave[r] = 1 + max(wave[q] for q in dests) if dests else 0
+    final = [max(0, min(sizes[r], total - B[r])) for r in range(G)]
+    return RebalancePlan(pieces, shift, kept, wave, final, total)
+
 
 @dataclass
 class ShardResult:
@@ -81,6 +153,7 @@ class ShardedDS:
         self.d_result = self.local.alloc_u64(2, self.device)
         self.d_entry = self.local.alloc_u64(1, self.device)
         self.d_halo = self.local.alloc_u64(self.world, self.device)
+        self._sizes = None  # every rank's shard capacity (rebalance), gathered once
 
     def _allgather(self, out: torch.Tensor, inp: torch.Tensor) -> None:
         if self.world == 1:
@@ -100,6 +173,37 @@ class ShardedDS:
     def select(self, shard: torch.Tensor, predicate: int, param: int = 0, stream=None) -> ShardResult:
         self.local.select(shard, predicate, param, self.d_count, stream)
         return self._finish(stream)
+
+    def rebalance(self, shard: torch.Tensor, res: ShardResult, stream=None) -> int:
+        """Contiguous global layout after a sharded compact/select/unique
+        (module docstring).  Returns the number of outputs this rank holds
+        at shard[0, ret); words past it are unspecified.  Host-synchronising
+        (the plan needs the counts on the host)."""
+        counts = [int(c) for c in res.counts.tolist()]
+        if self._sizes is None:
+            mine = torch.tensor([shard.numel()], dtype=torch.int64, device=self.device)
+            allsz = torch.zeros(self.world, dtype=torch.int64, device=self.device)
+            self._allgather(allsz, mine)
+            self._sizes = [int(x) for x in allsz.tolist()]
+        plan = rebalance_plan(counts, self._sizes)
+        me = self.rank
+        for w in range(plan.waves):
+            ops = []
+            if plan.wave[me] == w:
+                for pc in plan.pieces:
+                    if pc.src == me:
+                        ops.append(dist.P2POp(dist.isend, shard[pc.src_lo:pc.src_lo + pc.count],
+                                              pc.dst, self.group))
+            for pc in plan.pieces:
+                if pc.dst == me and plan.wave[pc.src] == w:
+                    ops.append(dist.P2POp(dist.irecv, shard[pc.dst_lo:pc.dst_lo + pc.count],
+                                          pc.src, self.group))
+            if ops:
+                for req in dist.batch_isend_irecv(ops):
+                    req.wait()
+            if plan.wave[me] == w and plan.shift[me] and plan.kept[me]:
+                self.local.slide(shard, counts[me], plan.shift[me], stream)
+        return plan.final[me]
 
     def unique(self, shard: torch.Tensor, stream=None) -> ShardResult:
         # Halo exchange before the slide (unique never changes a shard's last

@@ -27,6 +27,8 @@ SIGNATURES = {
     "ds_unpad": (_i, [_vp, _sz, _sz, _sz, _sz]),
     "ds_pad_ex": (_i, [_vp, _sz, _sz, _sz, _sz, _vp, _vp]),
     "ds_unpad_ex": (_i, [_vp, _sz, _sz, _sz, _sz, _vp]),
+    "ds_slide": (_i, [_vp, _sz, _sz, _sz]),
+    "ds_slide_ex": (_i, [_vp, _sz, _sz, _sz, _vp]),
     "ds_compact": (_i, [_vp, _sz, _u32, _psz]),
     "ds_select": (_i, [_vp, _sz, _i, _psz]),
     "ds_unique": (_i, [_vp, _sz, _psz]),
@@ -127,6 +129,14 @@ def ds_pad_ex(ptr, rows: int, cols: int, new_cols: int, elem_bytes: int,
 def ds_unpad_ex(ptr, rows: int, cols: int, new_cols: int, elem_bytes: int, stream=None) -> None:
     _check(_lib.ds_unpad_ex(_addr(ptr), rows, cols, new_cols, elem_bytes, _stream(stream)),
            "ds_unpad_ex")
+
+
+def ds_slide(ptr, n: int, shift: int, elem_bytes: int) -> None:
+    _check(_lib.ds_slide(_addr(ptr), n, shift, elem_bytes), "ds_slide")
+
+
+def ds_slide_ex(ptr, n: int, shift: int, elem_bytes: int, stream=None) -> None:
+    _check(_lib.ds_slide_ex(_addr(ptr), n, shift, elem_bytes, _stream(stream)), "ds_slide_ex")
 
 
 # -------------------------------------------------------------- irregular DS

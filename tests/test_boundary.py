@@ -134,3 +134,15 @@ def test_partition_and_copy_validation():
     assert st("ds_select_copy_ex", FAKE, 10, 0, 0, None, None, None) == INV  # no out
     assert st("ds_select_copy_ex", FAKE, 10, 0, 0, BAD, None, None) == INV   # misaligned out
     assert st("ds_partition_copy_ex", FAKE, 10, 0, 0, FAKE, None, None, None) == INV
+
+
+def test_slide_validation_before_device():
+    assert st("ds_slide_ex", FAKE, 10, 11, 4, None) == INV     # shift > n
+    assert st("ds_slide_ex", FAKE, 10, 1, 3, None) == INV      # bad elem_bytes
+    assert st("ds_slide_ex", FAKE, 10, 1, 2, None) == UNS      # 1/2-byte elements
+    assert st("ds_slide_ex", None, 10, 1, 4, None) == INV      # NULL with data
+    assert st("ds_slide_ex", BAD, 10, 1, 4, None) == INV       # misaligned
+    assert st("ds_slide_ex", FAKE, 1 << 62, 1, 16, None) == INV  # size overflow
+    assert st("ds_slide_ex", FAKE, 10, 0, 4, None) == 0         # nothing moves
+    assert st("ds_slide_ex", FAKE, 10, 10, 4, None) == 0        # nothing kept
+    assert st("ds_slide_ex", None, 0, 0, 4, None) == 0

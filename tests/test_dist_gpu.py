@@ -73,3 +73,41 @@ def test_sharded_ds_world1_on_gpu():
     torch.cuda.synchronize()
     assert int(res.count[0]) == m and res.result.tolist() == [0, m]
     assert np.array_equal(a.cpu().numpy().view(np.uint32), host)
+
+
+@pytest.mark.parametrize("G,fracs", [(2, [0.5, 0.5]), (4, [0.9, 0.1, 0.0, 1.0]), (8, [0.5] * 8),
+                                     (3, [0.0, 0.7, 0.2])])
+def test_fake_shard_rebalance(G, fracs):
+    """Rebalance plan executed on one GPU: the NCCL send/recv of each wave
+    replaced by device copies between the fake shards, the gap closed by the
+    real ds_slide kernel.  Result: the single-array in-place compaction."""
+    from paper_conf_icpp_gomez_lunacshg15_b200.dist import rebalance_plan
+    n = 2_000_003
+    parts = []
+    for i, f in enumerate(fracs):
+        lo, hi = shard_range(n, len(fracs), i)
+        parts.append(dsgen.compact_input(hi - lo, f, 50 + i, device="cuda"))
+    full = torch.cat(parts)
+    host = full.cpu().numpy().view(np.uint32).copy()
+    m = oracle.compact(host, 0)
+    shards, counts = [], torch.zeros(G, dtype=torch.int64, device="cuda")
+    for r in range(G):
+        lo, hi = shard_range(n, G, r)
+        shards.append(full[lo:hi])
+        libds.ds_compact_ex(full[lo:hi], hi - lo, 0, counts[r:r + 1], None)
+    c = [int(x) for x in counts.tolist()]
+    plan = rebalance_plan(c, [s.numel() for s in shards])
+    for w in range(plan.waves):
+        for r in range(G):
+            if plan.wave[r] != w:
+                continue
+            for pc in plan.pieces:
+                if pc.src == r:
+                    shards[pc.dst][pc.dst_lo:pc.dst_lo + pc.count].copy_(
+                        shards[r][pc.src_lo:pc.src_lo + pc.count])
+            if plan.shift[r] and plan.kept[r]:
+                libds.ds_slide_ex(shards[r], c[r], plan.shift[r], 4, None)
+    torch.cuda.synchronize()
+    got = full.cpu().numpy().view(np.uint32)
+    assert plan.total == m
+    assert np.array_equal(got[:m], host[:m])

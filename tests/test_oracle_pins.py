@@ -299,6 +299,44 @@ def test_unpad_equals_slicing():
     assert np.array_equal(buf[R * NC:], orig[R * NC:])
 
 
+def test_slide_brute_force_and_slicing():
+    """Every n <= 9, shift <= n, eb in {4, 8, 16}: numpy slicing closed form
+    (out[:n-shift] == in[shift:n]), untouched tail, buffer bytes past n."""
+    for eb in (4, 8, 16):
+        w = eb // 4
+        for n in range(0, 10):
+            for shift in range(0, n + 1):
+                buf = (np.arange(n * w + 3, dtype=np.uint32) * 2654435761) & 0xFFFFFFFF
+                buf = buf.astype(np.uint32)
+                orig = buf.copy()
+                oracle.slide(buf, n, shift, eb)
+                assert np.array_equal(buf[:(n - shift) * w], orig[shift * w:n * w]), (n, shift, eb)
+                assert np.array_equal(buf[(n - shift) * w:], orig[(n - shift) * w:])
+
+
+def test_slide_equals_unpad_of_two_rows():
+    """unpad(R=2, C, NC) moves row 1's first NC elements [C, C+NC) back by
+    C-NC to [NC, 2NC); a slide of the sub-buffer starting at element NC, with
+    n = C and shift = C-NC, makes the same move (cross-check of two oracle
+    functions written independently: memmove per row vs. element loop)."""
+    C, NC = 57, 40
+    a = dsgen.matrix_input(2, C, C, 4).numpy().view(np.uint32).copy()
+    b = a.copy()
+    oracle.unpad(a, 2, C, NC, 4)
+    sub = b[NC:2 * C].copy()          # elements NC .. 2C-1
+    oracle.slide(sub, C, C - NC, 4)  # sub[C-NC, C) -> sub[0, NC)
+    b[NC:2 * C] = sub
+    assert np.array_equal(a[:2 * NC], b[:2 * NC])
+
+
+def test_slide_invalid_args():
+    buf = np.zeros(8, dtype=np.uint32)
+    with pytest.raises(ValueError):
+        oracle.slide(buf, 4, 5, 4)
+    with pytest.raises(ValueError):
+        oracle.slide(buf, 4, 1, 0)
+
+
 def test_pad_default_fill_zero_and_row0_fixed():
     R, C, NC = 9, 10, 13
     buf = dsgen.matrix_input(R, C, NC, 4).numpy().view(np.uint32).copy()

@@ -367,3 +367,33 @@ def test_partition_copy_out_of_place(n):
     ot.assert_equals(et, "trues")
     of.assert_equals(ef, "falses")
     src.assert_equals(a, "input unchanged")
+
+
+# ---------------------------------------------------------------- slide
+@pytest.mark.parametrize("n,shift", [(1, 1), (2, 1), (5, 0), (9, 4), (T, 1), (3 * T + 7, 5),
+                                     (65537, 65536), (1_000_003, 3), (1_000_003, 12_345),
+                                     (1_000_003, 500_001), (300_000, 2 * 8192 + 1)])
+@pytest.mark.parametrize("eb", [4, 8, 16])
+@pytest.mark.parametrize("mis", [0, 1, 3])
+def test_slide(n, shift, eb, mis):
+    w = eb // 4
+    a = ((np.arange(n * w, dtype=np.uint64) * 2654435761 + 12345) & 0xFFFFFFFF).astype(np.uint32)
+    buf = DevBuf(a, mis)
+    exp = buf.host_region()
+    oracle.slide(exp, n, shift, eb)
+    libds.ds_slide(buf.ptr, n, shift, eb)
+    buf.assert_equals(exp, f"slide n={n} shift={shift} eb={eb} mis={mis}")
+
+
+def test_slide_ex_stream_repeated():
+    """Back-to-back slides on one stream (ticket/epoch re-arming across launches)."""
+    n = 200_003
+    a = dsgen.compact_input(n, 0.5, 99).numpy().view(np.uint32).copy()
+    buf = DevBuf(a, 2)
+    exp = buf.host_region()
+    s = torch.cuda.Stream()
+    for shift in (1, 7, 8192, 3, 40_000):
+        oracle.slide(exp, n, shift, 4)
+        libds.ds_slide_ex(buf.ptr, n, shift, 4, s)
+    s.synchronize()
+    buf.assert_equals(exp, "slide repeated")
