@@ -141,6 +141,24 @@ ds_status ds_unique_ex(void* ptr, size_t n, const uint64_t* d_halo,
                        size_t halo_len, uint64_t* d_out_n, ds_stream_t stream);
 
 /* ---------------------------------------------------------------------
+ * 8-byte elements (int64 / float64; the paper evaluates pad/unpad in double,
+ * P:220).  Same semantics as the 32-bit calls with n, values, counts
+ * in 8-byte ELEMENTS and equality on the 64-bit pattern (R13).  ptr must be
+ * 8-byte aligned.  ds_select64 takes the ds_predicate ids with the element
+ * type widened: I32_* compare as int64, F32_* as double (NaN -> false for
+ * GT, R16), EVEN/ODD test bit 0.  No shard halo for ds_unique64: its first
+ * element is always kept.
+ * ------------------------------------------------------------------- */
+ds_status ds_compact64(void* ptr, size_t n, uint64_t remove_value, size_t* out_n);
+ds_status ds_select64(void* ptr, size_t n, int predicate_id, size_t* out_n);
+ds_status ds_unique64(void* ptr, size_t n, size_t* out_n);
+ds_status ds_compact64_ex(void* ptr, size_t n, uint64_t remove_value,
+                          uint64_t* d_out_n, ds_stream_t stream);
+ds_status ds_select64_ex(void* ptr, size_t n, int predicate_id, uint64_t param,
+                         uint64_t* d_out_n, ds_stream_t stream);
+ds_status ds_unique64_ex(void* ptr, size_t n, uint64_t* d_out_n, ds_stream_t stream);
+
+/* ---------------------------------------------------------------------
  * Partition and out-of-place variants
  * ------------------------------------------------------------------- */
 
@@ -201,7 +219,7 @@ uint64_t ds_launch_count(void);
  * (globaltimer ns: 0 drawn, 1 landed, 2 aggregate published, 3 look-back
  * start, 4 prefix published, 5 stores start, 6 stores issued; 7 SM id;
  * 8 look-back rounds, 9 polls, 10 first round read, 11 resolved, 12 after
- * the acquire fence).
+ * the acquire fence; 13/14 ranker warp 0 before/after the ranker barrier).
  * NULL disables.  Development aid for DESIGN.md §7, not used by the API.  */
 ds_status ds_debug_set_trace(uint64_t* d_trace, size_t capacity_tiles);
 /* Library version, major*10000 + minor*100 + patch.                      */

@@ -63,6 +63,15 @@ def lib():
         L.oracle_pad.restype = i32
         L.oracle_unpad.argtypes = [vp, sz, sz, sz, sz]
         L.oracle_unpad.restype = i32
+        u64 = ctypes.c_uint64
+        L.oracle_predicate64.argtypes = [i32, u64, u64]
+        L.oracle_predicate64.restype = i32
+        L.oracle_compact64.argtypes = [vp, sz, u64]
+        L.oracle_compact64.restype = sz
+        L.oracle_select64.argtypes = [vp, sz, i32, u64]
+        L.oracle_select64.restype = sz
+        L.oracle_unique64.argtypes = [vp, sz]
+        L.oracle_unique64.restype = sz
         L.oracle_slide.argtypes = [vp, sz, sz, sz]
         L.oracle_slide.restype = i32
         _lib = L
@@ -168,3 +177,32 @@ def slide(buf: np.ndarray, n: int, shift: int, elem_bytes: int) -> None:
     rc = lib().oracle_slide(_ptr(buf), n, shift, elem_bytes)
     if rc != 0:
         raise ValueError("oracle_slide: shift > n or elem_bytes == 0")
+
+
+def _words64(a: np.ndarray) -> np.ndarray:
+    if a.dtype != np.uint64 or not a.flags.c_contiguous or not a.flags.writeable:
+        raise TypeError("oracle needs a writeable C-contiguous uint64 array")
+    return a
+
+
+def compact64(a: np.ndarray, remove_value: int) -> int:
+    """In place on uint64 ``a`` (8-byte elements); returns the kept count."""
+    a = _words64(a)
+    return int(lib().oracle_compact64(_ptr(a), a.size, remove_value & 0xFFFFFFFFFFFFFFFF))
+
+
+def select64(a: np.ndarray, pred: int, param: int = 0) -> int:
+    a = _words64(a)
+    r = lib().oracle_select64(_ptr(a), a.size, pred, param & 0xFFFFFFFFFFFFFFFF)
+    if r == ctypes.c_size_t(-1).value:
+        raise ValueError("unknown predicate")
+    return int(r)
+
+
+def unique64(a: np.ndarray) -> int:
+    a = _words64(a)
+    return int(lib().oracle_unique64(_ptr(a), a.size))
+
+
+def predicate64(pred: int, e: int, param: int = 0) -> int:
+    return int(lib().oracle_predicate64(pred, e & 0xFFFFFFFFFFFFFFFF, param & 0xFFFFFFFFFFFFFFFF))

@@ -139,3 +139,47 @@ int oracle_slide(uint8_t* b, size_t n, size_t shift, size_t elem_bytes) {
             b[(i - shift) * elem_bytes + k] = b[i * elem_bytes + k];
     return 0;
 }
+
+/* 8-byte elements: the same sequential definitions on 64-bit patterns. */
+int oracle_predicate64(int pred, uint64_t e, uint64_t param) {
+    double de, dp;
+    memcpy(&de, &e, sizeof de);
+    memcpy(&dp, &param, sizeof dp);
+    switch (pred) {
+    case ORACLE_PRED_NONZERO: return e != 0;
+    case ORACLE_PRED_I32_GT: return (int64_t)e > (int64_t)param;
+    case ORACLE_PRED_I32_NOT_GT: return !((int64_t)e > (int64_t)param);
+    case ORACLE_PRED_F32_GT: return de > dp;
+    case ORACLE_PRED_F32_NOT_GT: return !(de > dp);
+    case ORACLE_PRED_I32_EVEN: return (e & 1u) == 0;
+    case ORACLE_PRED_I32_ODD: return (e & 1u) != 0;
+    default: return -1;
+    }
+}
+
+size_t oracle_compact64(uint64_t* a, size_t n, uint64_t remove_value) {
+    size_t w = 0;
+    for (size_t i = 0; i < n; ++i)
+        if (a[i] != remove_value) a[w++] = a[i];
+    return w;
+}
+
+size_t oracle_select64(uint64_t* a, size_t n, int pred, uint64_t param) {
+    if (pred < 0 || pred >= ORACLE_PRED_COUNT) return (size_t)-1;
+    size_t w = 0;
+    for (size_t i = 0; i < n; ++i)
+        if (oracle_predicate64(pred, a[i], param)) a[w++] = a[i];
+    return w;
+}
+
+size_t oracle_unique64(uint64_t* a, size_t n) {
+    if (n == 0) return 0;
+    uint64_t prev = a[0];
+    size_t w = 1;
+    for (size_t i = 1; i < n; ++i) {
+        const uint64_t cur = a[i];
+        if (cur != prev) a[w++] = cur;
+        prev = cur;
+    }
+    return w;
+}

@@ -100,6 +100,16 @@ int oracle_pad(uint8_t* b, size_t rows, size_t cols, size_t new_cols,
 int oracle_unpad(uint8_t* b, size_t rows, size_t cols, size_t new_cols,
                  size_t elem_bytes);
 
+/* 8-byte elements (int64 / float64 bit patterns).  Same
+ * definitions as the 32-bit functions above with 64-bit elements: compaction
+ * removes elements bitwise-equal to the value; select keeps predicate-true
+ * elements, the predicate ids widened (I32 -> int64, F32 -> double, EVEN/ODD
+ * on bit 0); unique keeps element i iff i == 0 or a[i] != a[i-1].         */
+int oracle_predicate64(int pred, uint64_t e, uint64_t param);
+size_t oracle_compact64(uint64_t* a, size_t n, uint64_t remove_value);
+size_t oracle_select64(uint64_t* a, size_t n, int pred, uint64_t param);
+size_t oracle_unique64(uint64_t* a, size_t n);
+
 /* Slide, the one-group regular DS ("groups of consecutive input
  * array elements are shifted by a constant amount of memory positions"):
  * elements [shift, n) (elem_bytes each) move backward by `shift` to

@@ -166,6 +166,28 @@ ds_status run_regular(const ds::RegArgs& a, cudaStream_t s) {
     return e == cudaSuccess ? DS_SUCCESS : fail(e, "regular kernel launch");
 }
 
+// ---- 8-byte elements (n counts elements; the kernels see 2n words) ----
+ds_status check_wide(const void* ptr, size_t n, const uint64_t* d_out_n) {
+    if (n > 0 && ptr == nullptr) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(ptr, 8) || misaligned(d_out_n, 8)) return DS_ERROR_INVALID_VALUE;
+    if (n > kMaxWords / 2) return DS_ERROR_UNSUPPORTED;
+    return DS_SUCCESS;
+}
+
+ds::IrregArgs wide_args(void* ptr, size_t n, ds::IrregOp op, int pred, uint64_t value, uint64_t* d_out_n) {
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), 2 * n, op, pred, uint32_t(value), nullptr, 0, d_out_n};
+    a.wide = true;
+    a.value_hi = uint32_t(value >> 32);
+    return a;
+}
+
+ds_status wide_blocking(ds::IrregArgs a, size_t* out_n) {
+    size_t words = 0;
+    ds_status st = irregular_blocking(a, &words);  // the kernel reports elements already
+    if (st == DS_SUCCESS) *out_n = words;
+    return st;
+}
+
 ds_status sync_default() {
     cudaError_t e = cudaStreamSynchronize(nullptr);
     return e == cudaSuccess ? DS_SUCCESS : fail(e, "cudaStreamSynchronize");
@@ -400,6 +422,51 @@ ds_status ds_shard_offsets(const uint64_t* d_counts, size_t world, size_t rank, 
     cudaError_t e = ds::launch_shard_offsets(d_counts, world, rank, d_result,
                                              reinterpret_cast<cudaStream_t>(stream));
     return e == cudaSuccess ? DS_SUCCESS : fail(e, "shard offsets launch");
+}
+
+ds_status ds_compact64_ex(void* ptr, size_t n, uint64_t remove_value, uint64_t* d_out_n, ds_stream_t stream) {
+    ds_status st = check_wide(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    return irregular_ex(wide_args(ptr, n, ds::IrregOp::Compact, 0, remove_value, d_out_n),
+                        reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_select64_ex(void* ptr, size_t n, int predicate_id, uint64_t param, uint64_t* d_out_n,
+                         ds_stream_t stream) {
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_wide(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    return irregular_ex(wide_args(ptr, n, ds::IrregOp::Select, predicate_id, param, d_out_n),
+                        reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_unique64_ex(void* ptr, size_t n, uint64_t* d_out_n, ds_stream_t stream) {
+    ds_status st = check_wide(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    return irregular_ex(wide_args(ptr, n, ds::IrregOp::Unique, 0, 0, d_out_n),
+                        reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_compact64(void* ptr, size_t n, uint64_t remove_value, size_t* out_n) {
+    if (!out_n) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_wide(ptr, n, nullptr);
+    if (st != DS_SUCCESS) return st;
+    return wide_blocking(wide_args(ptr, n, ds::IrregOp::Compact, 0, remove_value, nullptr), out_n);
+}
+
+ds_status ds_select64(void* ptr, size_t n, int predicate_id, size_t* out_n) {
+    if (!out_n) return DS_ERROR_INVALID_VALUE;
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_wide(ptr, n, nullptr);
+    if (st != DS_SUCCESS) return st;
+    return wide_blocking(wide_args(ptr, n, ds::IrregOp::Select, predicate_id, 0, nullptr), out_n);
+}
+
+ds_status ds_unique64(void* ptr, size_t n, size_t* out_n) {
+    if (!out_n) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_wide(ptr, n, nullptr);
+    if (st != DS_SUCCESS) return st;
+    return wide_blocking(wide_args(ptr, n, ds::IrregOp::Unique, 0, 0, nullptr), out_n);
 }
 
 const char* ds_status_string(ds_status s) {

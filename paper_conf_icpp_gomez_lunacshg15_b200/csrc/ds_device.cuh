@@ -31,7 +31,7 @@ constexpr uint64_t kStateIncl = 2;    // irregular: inclusive prefix known
 // Status words are spread kStatusStride uint64 apart: tiles
 // finishing at the same time sit on different L2 lines.
 #ifndef DS_STATUS_STRIDE
-#define DS_STATUS_STRIDE 4
+#define DS_STATUS_STRIDE 8
 #endif
 constexpr uint64_t kStatusStride = DS_STATUS_STRIDE;
 __host__ __device__ __forceinline__ uint64_t* status_ptr(uint64_t* base, int64_t tile) {
@@ -159,6 +159,18 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // lets the hardware park the warp until the phase completes instead of
 // re-issuing try_wait in a tight loop.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+#ifdef DS_MBAR_SPIN
+    asm volatile(
+        "{\n"
+        ".reg .pred P;\n"
+        "DS_WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
+        "@!P bra DS_WAIT_%=;\n"
+        "}\n" ::"r"(smem_addr(bar)),
+        "r"(parity)
+        : "memory");
+    return;
+#endif
     asm volatile(
         "{\n"
         ".reg .pred P;\n"

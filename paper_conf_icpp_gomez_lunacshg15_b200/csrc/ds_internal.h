@@ -32,6 +32,8 @@ struct IrregArgs {
     uint64_t* d_out_n;  // may be null
     uint32_t* out_true = nullptr;   // kept / true words (null: in place at ptr)
     uint32_t* out_false = nullptr;  // false words in input order (null: dropped)
+    bool wide = false;              // 8-byte elements: n counts words (2 per element)
+    uint32_t value_hi = 0;          // high word of the 8-byte value / parameter
 };
 
 struct RegArgs {

@@ -53,6 +53,8 @@ struct IrregParams {
     uint32_t ntiles;
     uint32_t draws;   // ntiles + gridDim.x
     uint32_t value;   // compact: remove value; select: predicate parameter
+    uint32_t value_hi;  // 8-byte elements: high word of the value / parameter
+    uint32_t wshift;    // out_n = words >> wshift (1 for 8-byte elements)
     uint64_t* trace;  // diagnostics: per-tile events, or null
     uint32_t* tbase;  // 16-byte-aligned base of the true/kept output (== abase in place)
     uint64_t tlo;     // its word offset (output word j lives at tbase[tlo + j])
@@ -61,13 +63,16 @@ struct IrregParams {
 };
 
 // ---- predicates (a3) ----------------------------------------------------
+// kWide: the elements are 8 bytes (two consecutive words, the low word first);
+// both words of an element get the element's keep flag, so ranks, prefixes
+// and stores stay in words and every kept element moves as a pair.
 struct OpCompact {  // remove words equal to a value
-    static constexpr bool kUnique = false;
+    static constexpr bool kUnique = false, kWide = false;
     __device__ static bool keep(uint32_t w, uint32_t v) { return w != v; }
 };
 template <int P>
 struct OpSelect {  // keep predicate-true words (R14); ids = ds_predicate
-    static constexpr bool kUnique = false;
+    static constexpr bool kUnique = false, kWide = false;
     __device__ static bool keep(uint32_t w, uint32_t param) {
         if constexpr (P == 0) return w != 0u;
         else if constexpr (P == 1) return int32_t(w) > int32_t(param);
@@ -79,8 +84,29 @@ struct OpSelect {  // keep predicate-true words (R14); ids = ds_predicate
     }
 };
 struct OpUnique {  // keep w[i] iff it differs from w[i-1]
-    static constexpr bool kUnique = true;
+    static constexpr bool kUnique = true, kWide = false;
     __device__ static bool keep(uint32_t, uint32_t) { return true; }
+};
+// 8-byte elements: same primitives on int64 / float64 values.
+struct OpCompact64 {
+    static constexpr bool kUnique = false, kWide = true;
+    __device__ static bool keep2(uint64_t e, uint64_t v) { return e != v; }
+};
+template <int P>
+struct OpSelect64 {  // ds_predicate ids with the element type widened: I32 -> int64, F32 -> double
+    static constexpr bool kUnique = false, kWide = true;
+    __device__ static bool keep2(uint64_t e, uint64_t param) {
+        if constexpr (P == 0) return e != 0ull;
+        else if constexpr (P == 1) return int64_t(e) > int64_t(param);
+        else if constexpr (P == 2) return !(int64_t(e) > int64_t(param));
+        else if constexpr (P == 3) return __longlong_as_double(int64_t(e)) > __longlong_as_double(int64_t(param));
+        else if constexpr (P == 4) return !(__longlong_as_double(int64_t(e)) > __longlong_as_double(int64_t(param)));
+        else if constexpr (P == 5) return (e & 1ull) == 0ull;
+        else return (e & 1ull) != 0ull;
+    }
+};
+struct OpUnique64 {
+    static constexpr bool kUnique = true, kWide = true;
 };
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -96,9 +122,6 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 #ifndef DS_IRR_IN_STAGES
 #define DS_IRR_IN_STAGES 6
 #endif
-#ifndef DS_IRR_RING_WORDS
-#define DS_IRR_RING_WORDS 0
-#endif
 #ifndef DS_IRR_SLOTS
 #define DS_IRR_SLOTS 12
 #endif
@@ -108,11 +131,9 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 constexpr int kRankWarps = DS_IRR_RANK_WARPS;
 constexpr int kRT = 32 * kRankWarps;      // ranker threads
 constexpr int kSeg = 512;                 // contiguous words ranked by one warp
-constexpr int kGroup = 8;                 // contiguous words per lane per group
-constexpr int kGroups = kSeg / (32 * kGroup);  // groups per warp (2)
+constexpr int kChunks = kSeg / 32;        // 32-word chunks per warp segment (16)
 constexpr int kT = kRankWarps * kSeg;     // words per tile (8192 = 32 KB with 16 rankers)
 constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
-constexpr int kRingWords = DS_IRR_RING_WORDS; // compacted tiles awaiting their prefix (0: none)
 constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
 constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
 constexpr int kStoreWarps = 5;
@@ -127,49 +148,22 @@ constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;
 constexpr int kThreads = 32 * (kWarpProducer + 1);
 constexpr int kPre = 4;                   // words before the tile (unique's boundary word)
 constexpr int kStageWords = kT + kPre + 4;
-constexpr size_t kSmem = (size_t(kInStages) * kStageWords + kRingWords) * 4;
+constexpr size_t kSmem = size_t(kInStages) * kStageWords * 4;
 static_assert(kRankWarps <= 32, "warp-total scan in one warp");
 static_assert(kThreads <= 1024, "CTA size");
 static_assert(kSlots >= kInStages, "a slot per input stage at least");
 static_assert(kSlots % kResolvers == 0, "a slot is always served by the same resolver");
-static_assert(kRingWords % 4 == 0 && (kRingWords == 0 || kRingWords >= kT + 16),
-              "no ring, or a ring that holds one full tile");
 static_assert(kSmem <= 227 * 1024 - 4096, "shared memory");
 
-// Keep mask of the kGroup words w[] at tile word index x (from the staged
-// tile).
-template <class Op>
-__device__ __forceinline__ uint32_t keep_mask(const IrregParams& p, const uint32_t* stage,
-                                              uint64_t tb, bool full, int x, const uint32_t (&w)[kGroup],
-                                              bool has_hprev, uint32_t hprev) {
-    uint32_t m = 0;
-    if constexpr (Op::kUnique) {
-        uint32_t prev = stage[kPre + x - 1];  // x == 0: the word before the tile
-        const bool first = tb == 0 && x == 0;  // holds the array's first word (index p.lo < 4)
-#pragma unroll
-        for (int k = 0; k < kGroup; ++k) {
-            bool kp = w[k] != prev;
-            prev = w[k];
-            if (first && k == int(p.lo)) kp = !has_hprev || w[k] != hprev;  // shard halo (R18)
-            if (!full) {
-                const uint64_t e = tb + x + k;
-                kp = kp && e >= p.lo && e < p.hi;
-            }
-            m |= uint32_t(kp) << k;
-        }
-    } else {
-#pragma unroll
-        for (int k = 0; k < kGroup; ++k) {
-            bool kp = Op::keep(w[k], p.value);
-            if (!full) {
-                const uint64_t e = tb + x + k;
-                kp = kp && e >= p.lo && e < p.hi;
-            }
-            m |= uint32_t(kp) << k;
-        }
-    }
-    return m;
-}
+struct SlotMeta {
+    uint32_t tile;              // kNoTile: end of this CTA's work
+    uint32_t prev_tile;         // this CTA's previous ticket (kNoTile: none)
+    volatile uint32_t incl_tile;          // == tile once incl is valid (CTA-local chain)
+    volatile unsigned long long incl;     // inclusive prefix of the tile
+    uint32_t total;             // kept words in the tile
+    unsigned long long excl;    // kept words in all lower tiles
+    uint32_t wtot[kRankWarps];  // kept words in each ranker warp's segment
+};
 
 // Shard halo (R18): last word of the nearest non-empty earlier shard.
 __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) {
@@ -309,6 +303,92 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
     return excl;
 }
 
+#ifndef DS_IRR_LOCAL_CHAIN
+#define DS_IRR_LOCAL_CHAIN 0
+#endif
+constexpr bool kLocalChain = DS_IRR_LOCAL_CHAIN;
+#ifndef DS_IRR_LW
+#define DS_IRR_LW 8
+#endif
+constexpr int kLW = DS_IRR_LW;  // window slots per lane (32 * kLW tiles)
+
+// a5, CTA-local chain: this CTA's previous tile tp < t resolves first (its
+// resolver is in the same CTA), so t needs only the aggregates of the window
+// (tp, t) -- about one tile per other SM -- plus incl(tp) from shared memory,
+// or a nearer INCL inside the window.  One read of the window (<= 32*kLB
+// tiles), then only its pending slots are re-read; no multi-round walk.
+__device__ __forceinline__ uint64_t lookback_window(const uint64_t* __restrict__ status, uint32_t tile,
+                                                    uint32_t tp, const SlotMeta* pm, uint32_t epoch,
+                                                    int lane, uint64_t* trace) {
+    const uint32_t W = tile - tp - 1;  // window tiles tile-1 .. tp+1
+    const int64_t base = int64_t(tile) - 1;
+    uint64_t s[kLW];
+    uint32_t okm = 0;  // bit m: slot m current (or outside the window)
+#pragma unroll
+    for (int m = 0; m < kLW; ++m) {
+        const uint32_t d = uint32_t(32 * m + lane);
+        if (d < W) {
+            s[m] = ld_relaxed_gpu(status_ptr(status, base - d));
+            if (status_current(s[m], epoch)) okm |= 1u << m;
+        } else {
+            s[m] = 0;
+            okm |= 1u << m;
+        }
+    }
+    if (lane == 0) trace_event(trace, tile, 10, globaltimer());
+    uint32_t ns = kPollMinNs, polls = 0;
+    uint32_t M, L;
+    bool local;
+    while (true) {
+        uint32_t inclm = 0;
+#pragma unroll
+        for (int m = 0; m < kLW; ++m)
+            if (uint32_t(32 * m + lane) < W && (okm >> m & 1u) && status_state(s[m]) == kStateIncl) inclm |= 1u << m;
+        M = __reduce_min_sync(kFull, inclm ? uint32_t(__ffs(inclm) - 1) : uint32_t(kLW));
+        L = M < kLW ? uint32_t(__ffs(__ballot_sync(kFull, inclm >> M & 1u)) - 1) : 32u;
+        const uint32_t need = (M < kLW ? ((1u << M) - 1u) : ((1u << kLW) - 1u)) |
+                              (M < kLW && uint32_t(lane) <= L ? (1u << M) : 0u);
+        const bool have = !__any_sync(kFull, (okm & need) != need);
+        local = M == kLW && __shfl_sync(kFull, pm->incl_tile, 0) == tp;
+        if (have && (M < kLW || local)) break;
+        __nanosleep(ns);
+        ns = ns < kPollMaxNs ? ns * 2 : kPollMaxNs;
+        ++polls;
+#pragma unroll
+        for (int m = 0; m < kLW; ++m) {
+            const bool pending = !(okm >> m & 1u);
+            const bool refresh = m < kRefreshRows && !pending && status_state(s[m]) != kStateIncl;
+            if ((need >> m & 1u) && (pending || (refresh && !local))) {
+                const int64_t idx = base - (32 * m + lane);
+                if (uint32_t(32 * m + lane) < W) {
+                    s[m] = ld_relaxed_gpu(status_ptr(status, idx));
+                    okm = status_current(s[m], epoch) ? (okm | 1u << m) : (okm & ~(1u << m));
+                }
+            }
+        }
+    }
+    uint32_t agg = 0;
+    uint64_t inc = 0;
+#pragma unroll
+    for (int m = 0; m < kLW; ++m) {
+        const bool inw = uint32_t(32 * m + lane) < W;
+        if (inw && (uint32_t(m) < M || (uint32_t(m) == M && uint32_t(lane) < L))) agg += uint32_t(status_count(s[m]));
+        if (uint32_t(m) == M && uint32_t(lane) == L) inc = status_count(s[m]);
+    }
+    uint64_t excl = uint64_t(__reduce_add_sync(kFull, agg));
+    __threadfence_block();  // incl was written before incl_tile
+    excl += M < kLW ? __shfl_sync(kFull, inc, L) : pm->incl;
+    if (lane == 0) {
+        trace_event(trace, tile, 8, M < kLW ? 1 : 0);
+        trace_event(trace, tile, 9, polls);
+        trace_event(trace, tile, 11, globaltimer());
+    }
+    lookback_acquire();
+    __syncwarp();
+    if (lane == 0) trace_event(trace, tile, 12, globaltimer());
+    return excl;
+}
+
 // a7 helper: write the `cnt` words stage[src_off, src_off + cnt) to the
 // output words base[d0, d0 + cnt) (virtual indices; base is 16-byte aligned).
 // Destination chunks of 4 aligned words are read as two aligned shared
@@ -395,16 +475,6 @@ __device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph
     }
 }
 
-struct SlotMeta {
-    uint32_t tile;              // kNoTile: end of this CTA's work
-    uint32_t total;             // kept words in the tile
-    unsigned long long excl;    // kept words in all lower tiles
-    uint32_t ring_base;         // ring word index of rank 0 (multiple of 4, >= 4)
-    uint32_t ring_end;          // ring allocation counter after this tile
-    uint32_t in_ring;           // compacted into the ring (else in place in its input stage)
-    uint32_t tail_snap;         // ring tail seen before the decision
-    uint32_t wtot[kRankWarps];  // kept words in each ranker warp's segment
-};
 
 // mbarrier wait that also returns (false) once the CTA's work is known to
 // end before ring position k (the resolvers take alternate positions, so the
@@ -422,14 +492,12 @@ __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
 template <class Op, bool PART>
 __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParams p) {
     extern __shared__ __align__(128) uint32_t smem[];
-    uint32_t* const ring = smem + kInStages * kStageWords;
     __shared__ __align__(8) uint64_t bar_full[kInStages], bar_free[kInStages];
     __shared__ __align__(8) uint64_t bar_drawn[kSlots], bar_counted[kSlots], bar_ranked[kSlots],
         bar_resolved[kSlots], bar_stored[kSlots];
     __shared__ SlotMeta meta[kSlots];
     __shared__ uint32_t s_epoch;
     __shared__ volatile uint32_t s_end;        // ring position of the end marker
-    __shared__ volatile uint32_t s_ring_tail;  // ring words released by the storers (monotone)
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
@@ -445,7 +513,6 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             mbar_init(&bar_stored[o], 1);
         }
         s_end = 0xffffffffu;
-        s_ring_tail = 0;
         mbar_fence_init();
     }
     __syncthreads();
@@ -453,6 +520,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
     if (warp == kWarpProducer) {
         // ------------------------------------------------ producer (lane 0)
         if (lane != 0) return;
+        uint32_t prev_t = kNoTile;
         for (uint32_t k = 0;; ++k) {
             const int s = k % kInStages, o = k % kSlots;
             uint32_t* stage = smem + s * kStageWords;
@@ -469,6 +537,8 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 return;
             }
             meta[o].tile = t;
+            meta[o].prev_tile = prev_t;
+            prev_t = t;
             mbar_arrive(&bar_drawn[o]);  // the resolver starts this tile's look-back now
             trace_event(p.trace, t, 0, globaltimer());
             trace_event(p.trace, t, 7, smid());
@@ -476,11 +546,15 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint64_t tb = uint64_t(t) * kT;
             uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
             end = (end + 3) & ~3ull;  // may read <= 12 bytes past the array end (same 16 B chunk)
-            const uint64_t beg = (Op::kUnique && t > 0) ? tb - 4 : tb;
-            const uint32_t bytes = uint32_t(end - beg) * 4u;
+            // The tile itself from its 128-byte aligned start; unique's 16 bytes
+            // before it as a second copy (one unaligned copy would touch an extra
+            // line per request block).
+            const bool pre = Op::kUnique && t > 0;
+            const uint32_t bytes = uint32_t(end - tb) * 4u;
             fence_proxy_async_smem();
-            mbar_arrive_expect_tx(&bar_full[s], bytes);
-            bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_full[s]);
+            mbar_arrive_expect_tx(&bar_full[s], bytes + (pre ? 16u : 0u));
+            if (pre) bulk_g2s(stage, p.abase + tb - kPre, 16u, &bar_full[s]);
+            bulk_g2s(stage + kPre, p.abase + tb, bytes, &bar_full[s]);
         }
     } else if (warp < kRankWarps) {
         // ------------------------------------------------ ranker warps
@@ -489,7 +563,6 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         bool has_hprev = false;
         uint32_t hprev = 0;
         if (Op::kUnique) has_hprev = halo_prev(p, hprev);
-        uint32_t ring_head = 0;  // output-ring allocation counter (monotone, words; same in every warp)
         for (uint32_t k = 0;; ++k) {
             const int s = k % kInStages, o = k % kSlots;
             uint32_t* stage = smem + s * kStageWords;
@@ -500,35 +573,49 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint64_t tb = uint64_t(t) * kT;
             const bool full = tb >= p.lo && tb + kT <= p.hi;
 
-            // a3/a4: warp rw ranks tile words [kSeg*rw, kSeg*(rw+1)); in group g
-            // lane l holds the kGroup contiguous words at x = kSeg*rw + 256g + 8l.
-            uint32_t v[kGroups][kGroup];
-            uint32_t masks = 0;     // kGroup keep bits per group
-            uint32_t lane_pre = 0;  // 16 bits per group: kept words of lower lanes
-            uint32_t wrun = 0;      // kept words of the warp's earlier groups
-            uint32_t goff = 0;      // 16 bits per group: offset of group g in the segment
+            // a3/a4: warp rw ranks tile words [xs, xs + kSeg) in kChunks chunks of
+            // 32: lane l holds word x = xs + 32c + l of chunk c, so every shared
+            // load and every compaction store below touches 32 consecutive words
+            // (no bank conflicts), and a chunk's keep flags are one ballot.
+            const int xs = kSeg * rw;
+            uint32_t v[kChunks], mk[kChunks];
+            uint32_t wrun = 0;  // kept words of the warp's segment
 #pragma unroll
-            for (int g = 0; g < kGroups; ++g) {
-                const int x = kSeg * rw + 32 * kGroup * g + kGroup * lane;
-                const u32x4 q0 = *reinterpret_cast<const u32x4*>(stage + kPre + x);
-                const u32x4 q1 = *reinterpret_cast<const u32x4*>(stage + kPre + x + 4);
-                v[g][0] = q0.x; v[g][1] = q0.y; v[g][2] = q0.z; v[g][3] = q0.w;
-                v[g][4] = q1.x; v[g][5] = q1.y; v[g][6] = q1.z; v[g][7] = q1.w;
-                const uint32_t m = keep_mask<Op>(p, stage, tb, full, x, v[g], has_hprev, hprev);
-                masks |= m << (kGroup * g);
-                const uint32_t c = __popc(m);  // 0..8
-                const uint32_t b0 = __ballot_sync(kFull, c & 1u);
-                const uint32_t b1 = __ballot_sync(kFull, c & 2u);
-                const uint32_t b2 = __ballot_sync(kFull, c & 4u);
-                const uint32_t b3 = __ballot_sync(kFull, c & 8u);
-                lane_pre |= (__popc(b0 & lt) + 2u * __popc(b1 & lt) + 4u * __popc(b2 & lt) +
-                             8u * __popc(b3 & lt)) << (16 * g);
-                goff |= wrun << (16 * g);
-                wrun += __popc(b0) + 2u * __popc(b1) + 4u * __popc(b2) + 8u * __popc(b3);
+            for (int c = 0; c < kChunks; ++c) v[c] = stage[kPre + xs + 32 * c + lane];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                const int x = xs + 32 * c + lane;
+                bool kp;
+                if constexpr (Op::kWide) {
+                    // element = (even word, odd word) = lanes (2m, 2m+1) of the chunk
+                    const uint32_t partner = __shfl_xor_sync(kFull, v[c], 1);
+                    const uint32_t lo = (lane & 1) ? partner : v[c], hi = (lane & 1) ? v[c] : partner;
+                    const int xe = x - (lane & 1);  // the element's first word
+                    if constexpr (Op::kUnique) {
+                        kp = lo != stage[kPre + xe - 2] || hi != stage[kPre + xe - 1];
+                        if (tb + xe == p.lo) kp = true;  // the array's first element
+                    } else {
+                        kp = Op::keep2((uint64_t(hi) << 32) | lo, (uint64_t(p.value_hi) << 32) | p.value);
+                    }
+                } else if constexpr (Op::kUnique) {
+                    // previous word straight from the staged tile; x == 0 reads
+                    // the word before the tile
+                    kp = v[c] != stage[kPre + x - 1];
+                    if (tb + x == p.lo) kp = !has_hprev || v[c] != hprev;  // the array's first word (R18)
+                } else {
+                    kp = Op::keep(v[c], p.value);
+                }
+                if (!full) {
+                    const uint64_t e = tb + x;
+                    kp = kp && e >= p.lo && e < p.hi;
+                }
+                mk[c] = __ballot_sync(kFull, kp);
+                wrun += __popc(mk[c]);
             }
             if (lane == 0) meta[o].wtot[rw] = wrun;
-            if (rt == 0) meta[o].tail_snap = s_ring_tail;  // the ring tail only grows
-            named_bar_sync(1, kRT);  // warp totals + tail snapshot written; every ranker holds its words
+            if (rt == 0) trace_event(p.trace, t, 13, globaltimer());
+            named_bar_sync(1, kRT);  // warp totals written; every ranker holds its words
+            if (rt == 0) trace_event(p.trace, t, 14, globaltimer());
 
             // Exclusive scan of the kRankWarps warp totals (input order), redundantly
             // in every warp.
@@ -541,63 +628,39 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             }
             const uint32_t total = __shfl_sync(kFull, iw, 31);
             const uint32_t wbase = __shfl_sync(kFull, iw - cw, rw);
-            // Where to compact: into the output ring if the tile fits against the
-            // tail snapshot (then the input stage is free at once), else in place in
-            // the input stage (the storers free it).  Never waiting here keeps every
-            // drawn tile's AGG independent of other tiles.  Ring allocation:
-            // [4 slack | total rounded up to 4 | 4 slack], contiguous (skip to the
-            // start rather than wrap).  Every warp computes the same decision and
-            // allocation from the same values, so no further barrier is needed.
-            const uint32_t need = 8u + ((total + 3u) & ~3u);
-            const uint32_t pos = kRingWords ? ring_head % kRingWords : 0u;
-            const uint32_t skip = pos + need > uint32_t(kRingWords) ? uint32_t(kRingWords) - pos : 0u;
-            // (partition keeps the whole tile -- trues, then falses -- in its stage)
-            const bool in_ring = !PART && kRingWords > 0 &&
-                                 ring_head + skip + need - meta[o].tail_snap <= uint32_t(kRingWords);
-            uint32_t base = kPre;
-            if (in_ring) {
-                base = (ring_head + skip) % (kRingWords ? kRingWords : 1) + 4u;
-                ring_head += skip + need;
-            }
-            if (rt == 0 && in_ring) mbar_arrive(&bar_free[s]);  // the input stage may be refilled
             if (rt == 0) {
                 // a4: publish the aggregate right away -- it depends on nothing else
                 // (a relaxed status store).
                 meta[o].total = total;
-                meta[o].ring_base = base;
-                meta[o].ring_end = ring_head;
-                meta[o].in_ring = in_ring;
                 debug_delay(t, 1);
                 publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
                 trace_event(p.trace, t, 2, globaltimer());
                 mbar_arrive(&bar_counted[o]);
             }
 
-            // a6: compact the kept words: rank r -> ring[base + r], or in place
-            // -> stage[kPre + r] (every ranker's words are in registers).
+            // a6: compact the kept words in place, rank r -> stage[kPre + r]
+            // (every ranker's words are in registers since the barrier).
             // Partition also places the false words, in input order, after the
             // trues: the f-th false word goes to stage[kPre + total + f], where
             // f = (valid words before it in the tile) - (true words before it).
-            uint32_t* out = (in_ring ? ring : stage) + base;
+            uint32_t* out = stage + kPre;
             const uint32_t vstart = tb < p.lo ? uint32_t(p.lo - tb) : 0u;  // invalid lead words (tile 0)
+            uint32_t r = wbase;
 #pragma unroll
-            for (int g = 0; g < kGroups; ++g) {
-                uint32_t r = wbase + ((goff >> (16 * g)) & 0xFFFFu) + ((lane_pre >> (16 * g)) & 0xFFFFu);
-                const uint32_t m = masks >> (kGroup * g);
-                const int x = kSeg * rw + 32 * kGroup * g + kGroup * lane;
-#pragma unroll
-                for (int kk = 0; kk < kGroup; ++kk) {
-                    if (m >> kk & 1u) {
-                        out[r++] = v[g][kk];
-                    } else if (PART) {
-                        const uint64_t e = tb + x + kk;
-                        if (e >= p.lo && e < p.hi) out[total + (uint32_t(x + kk) - vstart) - r] = v[g][kk];
-                    }
+            for (int c = 0; c < kChunks; ++c) {
+                const uint32_t rl = r + __popc(mk[c] & lt);  // trues before this word in the tile
+                if (mk[c] >> lane & 1u) {
+                    out[rl] = v[c];
+                } else if (PART) {
+                    const uint32_t x = uint32_t(xs + 32 * c + lane);
+                    const uint64_t e = tb + x;
+                    if (e >= p.lo && e < p.hi) out[total + (x - vstart) - rl] = v[c];
                 }
+                r += __popc(mk[c]);
             }
-            fence_proxy_async_smem();  // the compacted words may leave through a bulk store
+            fence_proxy_async_smem();  // the compacted words leave through a bulk store
             __syncwarp();
-            if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is in the ring
+            if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is compacted
         }
     } else if (warp < kWarpStorer0) {
         // ------------------------------------------------ resolver warps
@@ -622,17 +685,28 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
 #ifdef DS_DEBUG_NO_LOOKBACK  // timing experiment only: wrong output, same traffic
             const uint64_t excl = uint64_t(t) * (kT / 2);
 #else
-            const uint64_t excl = t > 0 ? lookback(p.status, t, epoch, lane, p.trace) : 0ull;
+            uint64_t excl = 0;
+            if (t > 0) {
+                const uint32_t tp = meta[o].prev_tile;
+                if (kLocalChain && tp != kNoTile && t - tp - 1 <= uint32_t(32 * kLW))
+                    excl = lookback_window(p.status, t, tp, &meta[(k + kSlots - 1) % kSlots], epoch, lane, p.trace);
+                else
+                    excl = lookback(p.status, t, epoch, lane, p.trace);
+            }
 #endif
             mbar_wait(&bar_counted[o], use & 1);  // the tile's aggregate is published
             const uint32_t total = meta[o].total;
-            if (lane == 0 && t > 0)
-                publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
-            mbar_wait(&bar_ranked[o], use & 1);  // the compacted tile is in the ring
+            if (lane == 0) {
+                meta[o].incl = excl + total;  // the CTA's next tile chains on this
+                __threadfence_block();
+                meta[o].incl_tile = t;
+                if (t > 0) publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
+            }
+            mbar_wait(&bar_ranked[o], use & 1);  // the compacted tile is in its stage
             if (lane == 0) {
                 trace_event(p.trace, t, 4, globaltimer());
                 meta[o].excl = excl;
-                if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = excl + total;
+                if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = (excl + total) >> p.wshift;
                 mbar_arrive(&bar_resolved[o]);
             }
         }
@@ -641,17 +715,10 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         // a7.  Kept words go out through one TMA bulk store per tile (the
         // aligned interior) plus <= 6 scalar head/tail words.  The stage is
         // first re-phased in shared memory so that its words sit at the same
-        // 16-byte phase as their destination.  A tile's stage is released
-        // kStoreLag tiles later, once the bulk engine has finished reading it.
-        // Partition (two destinations) keeps the register path (store_segment).
+        // 16-byte phase as their destination; the stage is released once the
+        // bulk engine has read it.  Partition (two destinations) keeps the
+        // register path (store_segment).
         const int st = tid - 32 * kWarpStorer0;
-        int pend_s = -1, pend_o = -1;  // the tile whose release is pending (lag 1)
-        uint32_t pend_ring = 0, pend_in_ring = 0;
-        auto release = [&](int s_in, int o, uint32_t in_ring, uint32_t ring_end) {
-            if (in_ring) s_ring_tail = ring_end;
-            else mbar_arrive(&bar_free[s_in]);  // the in-place tile's input stage is free
-            mbar_arrive(&bar_stored[o]);
-        };
         for (uint32_t k = 0;; ++k) {
             const int o = k % kSlots;
             mbar_wait(&bar_resolved[o], (k / kSlots) & 1);
@@ -661,74 +728,52 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 trace_event(p.trace, t, 5, globaltimer());
                 debug_delay(t, 3);
             }
-            // a7: the kept words -> [excl, excl + A) of the true output; for a
-            // partition also the false words -> [excl_false, ...) of the false output.
-            const uint32_t in_ring = meta[o].in_ring;
             const int s_in = k % kInStages;
-            uint32_t* buf = in_ring ? ring : smem + s_in * kStageWords;
-            const int32_t rb = int32_t(meta[o].ring_base);
+            uint32_t* const seg = smem + s_in * kStageWords + kPre;  // rank 0 (16-byte aligned)
             const uint32_t A = meta[o].total;
             const uint64_t tb0 = uint64_t(t) * kT;
             const uint64_t vs0 = tb0 > p.lo ? tb0 : p.lo;
             const uint64_t ve0 = tb0 + kT < p.hi ? tb0 + kT : p.hi;
+            // Identity tile (in place, nothing removed in or before it): every
+            // kept word would be written onto itself, so the stores are skipped.
+            const bool identity = !PART && p.tbase == p.abase && meta[o].excl == vs0 - p.lo && A == ve0 - vs0;
 #ifndef DS_DEBUG_NO_STORE  // timing experiment only: no output written
             if (PART || !kBulkStore) {
-                if (!PART && p.tbase == p.abase && meta[o].excl == vs0 - p.lo && A == ve0 - vs0) {
-                    // identity tile: nothing to store
-                } else {
-                    store_segment<kST>(p.tbase, p.tlo + meta[o].excl, A, buf, rb, st);
-                }
+                if (!identity) store_segment<kST>(p.tbase, p.tlo + meta[o].excl, A, seg, 0, st);
                 if (PART) {
                     const uint64_t excl_f = (vs0 - p.lo) - meta[o].excl;
-                    store_segment<kST>(p.fbase, p.flo + excl_f, uint32_t(ve0 - vs0) - A, buf, rb + int32_t(A), st);
+                    store_segment<kST>(p.fbase, p.flo + excl_f, uint32_t(ve0 - vs0) - A, seg, int32_t(A), st);
                 }
-            } else {
-                // Identity tile (in place, nothing removed in or before it): every
-                // kept word would be written onto itself, so the stores are skipped.
-                const bool identity = p.tbase == p.abase && meta[o].excl == vs0 - p.lo && A == ve0 - vs0;
-                if (!identity && A > 0) {
-                    const uint64_t d0 = p.tlo + meta[o].excl, d1 = d0 + A;
-                    const uint32_t ph = uint32_t(d0) & 3u;
-                    uint32_t* seg = buf + rb;  // 16-byte aligned (rb % 4 == 0)
-                    if (ph) rephase<kST>(seg, A, ph, st);  // word r -> seg[ph + r]
-                    const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
-                    if (g1 > g0) {
-                        fence_proxy_async_smem();  // re-phased words -> visible to the bulk engine
-                        named_bar_sync(2, kST);
-                        if (st == 0)
-                            bulk_s2g(p.tbase + g0, seg + ph + uint32_t(g0 - d0), uint32_t(g1 - g0) * 4u);
-                        // head [d0, g0) and tail [g1, d1): at most 3 words each
-                        if (st < 3 && d0 + st < g0) stg_stream(p.tbase + d0 + st, seg[ph + st]);
-                        if (st >= 3 && st < 6 && g1 + (st - 3) < d1)
-                            stg_stream(p.tbase + g1 + (st - 3), seg[ph + uint32_t(g1 - d0) + (st - 3)]);
-                    } else {
-                        named_bar_sync(2, kST);
-                        if (uint32_t(st) < A) stg_stream(p.tbase + d0 + st, seg[ph + st]);  // A < 8
-                    }
+            } else if (!identity && A > 0) {
+                const uint64_t d0 = p.tlo + meta[o].excl, d1 = d0 + A;
+                const uint32_t ph = uint32_t(d0) & 3u;
+                if (ph) rephase<kST>(seg, A, ph, st);  // word r -> seg[ph + r]
+                const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
+                if (g1 > g0) {
+                    fence_proxy_async_smem();  // re-phased words -> visible to the bulk engine
+                    named_bar_sync(2, kST);
+                    if (st == 0)
+                        bulk_s2g(p.tbase + g0, seg + ph + uint32_t(g0 - d0), uint32_t(g1 - g0) * 4u);
+                    // head [d0, g0) and tail [g1, d1): at most 3 words each
+                    if (st < 3 && d0 + st < g0) stg_stream(p.tbase + d0 + st, seg[ph + st]);
+                    if (st >= 3 && st < 6 && g1 + (st - 3) < d1)
+                        stg_stream(p.tbase + g1 + (st - 3), seg[ph + uint32_t(g1 - d0) + (st - 3)]);
+                } else {
+                    named_bar_sync(2, kST);
+                    if (uint32_t(st) < A) stg_stream(p.tbase + d0 + st, seg[ph + st]);  // A < 8
                 }
             }
 #endif
-            named_bar_sync(2, kST);  // every storer is done reading the tile's stage
+            named_bar_sync(2, kST);  // every storer is done reading the stage
             if (st == 0) {
                 trace_event(p.trace, t, 6, globaltimer());
-                bulk_commit();  // (possibly empty) group of this tile
-                if (PART || !kBulkStore) {
-                    release(s_in, o, in_ring, meta[o].ring_end);
-                } else {
-                    bulk_wait_read<1>();  // the previous tile's stage has been read
-                    if (pend_o >= 0) release(pend_s, pend_o, pend_in_ring, pend_ring);
-                    pend_s = s_in;
-                    pend_o = o;
-                    pend_in_ring = in_ring;
-                    pend_ring = meta[o].ring_end;
-                }
+                bulk_commit();        // (possibly empty) group of this tile
+                bulk_wait_read<0>();  // the bulk engine has read the stage
+                mbar_arrive(&bar_free[s_in]);
+                mbar_arrive(&bar_stored[o]);
             }
         }
-        if (st == 0) {
-            bulk_wait_read<0>();
-            if (pend_o >= 0) release(pend_s, pend_o, pend_in_ring, pend_ring);
-            bulk_wait_all();  // the bulk stores are complete before the CTA exits
-        }
+        if (st == 0) bulk_wait_all();  // the bulk stores are complete before the CTA exits
     }
 }
 
@@ -782,6 +827,8 @@ cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s) 
     p.halo_len = uint32_t(a.halo_len);
     p.ntiles = uint32_t(irregular_tiles(a));
     p.value = a.value;
+    p.value_hi = a.value_hi;
+    p.wshift = a.wide ? 1u : 0u;
     p.trace = debug_trace(p.ntiles);
     uint32_t* tptr = a.out_true ? a.out_true : a.ptr;
     const uint64_t tmis = (reinterpret_cast<uintptr_t>(tptr) >> 2) & 3u;
@@ -794,6 +841,24 @@ cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s) 
     }
     count_launch();
     const bool part = a.out_false != nullptr;
+    if (a.wide) {
+        switch (a.op) {
+        case IrregOp::Compact: return launch_op<OpCompact64>(p, s);
+        case IrregOp::Unique: return launch_op<OpUnique64>(p, s);
+        case IrregOp::Select:
+            switch (a.predicate) {
+            case 0: return launch_op<OpSelect64<0>>(p, s);
+            case 1: return launch_op<OpSelect64<1>>(p, s);
+            case 2: return launch_op<OpSelect64<2>>(p, s);
+            case 3: return launch_op<OpSelect64<3>>(p, s);
+            case 4: return launch_op<OpSelect64<4>>(p, s);
+            case 5: return launch_op<OpSelect64<5>>(p, s);
+            case 6: return launch_op<OpSelect64<6>>(p, s);
+            default: return cudaErrorInvalidValue;
+            }
+        }
+        return cudaErrorInvalidValue;
+    }
     switch (a.op) {
     case IrregOp::Compact: return launch_op<OpCompact>(p, s);
     case IrregOp::Unique: return launch_op<OpUnique>(p, s);

@@ -35,6 +35,12 @@ SIGNATURES = {
     "ds_compact_ex": (_i, [_vp, _sz, _u32, _vp, _vp]),
     "ds_select_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp]),
     "ds_unique_ex": (_i, [_vp, _sz, _vp, _sz, _vp, _vp]),
+    "ds_compact64": (_i, [_vp, _sz, _u64, _psz]),
+    "ds_select64": (_i, [_vp, _sz, _i, _psz]),
+    "ds_unique64": (_i, [_vp, _sz, _psz]),
+    "ds_compact64_ex": (_i, [_vp, _sz, _u64, _vp, _vp]),
+    "ds_select64_ex": (_i, [_vp, _sz, _i, _u64, _vp, _vp]),
+    "ds_unique64_ex": (_i, [_vp, _sz, _vp, _vp]),
     "ds_partition": (_i, [_vp, _sz, _i, _vp, _psz]),
     "ds_partition_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp, _vp]),
     "ds_select_copy_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp, _vp]),
@@ -174,6 +180,40 @@ def ds_unique_ex(ptr, n: int, d_halo=None, halo_len: int = 0, d_out_n=None, stre
 
 
 # ------------------------------------------------- partition / out-of-place
+# ------------------------------------------------------- 8-byte elements
+def ds_compact64(ptr, n: int, remove_value: int) -> int:
+    out = ctypes.c_size_t(0)
+    _check(_lib.ds_compact64(_addr(ptr), n, remove_value & 0xFFFFFFFFFFFFFFFF, ctypes.byref(out)),
+           "ds_compact64")
+    return out.value
+
+
+def ds_select64(ptr, n: int, predicate_id: int) -> int:
+    out = ctypes.c_size_t(0)
+    _check(_lib.ds_select64(_addr(ptr), n, predicate_id, ctypes.byref(out)), "ds_select64")
+    return out.value
+
+
+def ds_unique64(ptr, n: int) -> int:
+    out = ctypes.c_size_t(0)
+    _check(_lib.ds_unique64(_addr(ptr), n, ctypes.byref(out)), "ds_unique64")
+    return out.value
+
+
+def ds_compact64_ex(ptr, n: int, remove_value: int, d_out_n=None, stream=None) -> None:
+    _check(_lib.ds_compact64_ex(_addr(ptr), n, remove_value & 0xFFFFFFFFFFFFFFFF, _addr(d_out_n),
+                                _stream(stream)), "ds_compact64_ex")
+
+
+def ds_select64_ex(ptr, n: int, predicate_id: int, param: int = 0, d_out_n=None, stream=None) -> None:
+    _check(_lib.ds_select64_ex(_addr(ptr), n, predicate_id, param & 0xFFFFFFFFFFFFFFFF, _addr(d_out_n),
+                               _stream(stream)), "ds_select64_ex")
+
+
+def ds_unique64_ex(ptr, n: int, d_out_n=None, stream=None) -> None:
+    _check(_lib.ds_unique64_ex(_addr(ptr), n, _addr(d_out_n), _stream(stream)), "ds_unique64_ex")
+
+
 def ds_partition(ptr, n: int, predicate_id: int, aux) -> int:
     out = ctypes.c_size_t(0)
     _check(_lib.ds_partition(_addr(ptr), n, predicate_id, _addr(aux), ctypes.byref(out)), "ds_partition")

@@ -146,3 +146,14 @@ def test_slide_validation_before_device():
     assert st("ds_slide_ex", FAKE, 10, 0, 4, None) == 0         # nothing moves
     assert st("ds_slide_ex", FAKE, 10, 10, 4, None) == 0        # nothing kept
     assert st("ds_slide_ex", None, 0, 0, 4, None) == 0
+
+
+def test_wide_validation_before_device():
+    assert st("ds_compact64_ex", BAD, 10, 0, None, None) == INV          # 4-byte aligned only
+    assert st("ds_compact64_ex", FAKE + 4, 10, 0, None, None) == INV     # not 8-byte aligned
+    assert st("ds_compact64_ex", None, 10, 0, None, None) == INV
+    assert st("ds_select64_ex", FAKE, 10, 9, 0, None, None) == INV       # bad predicate
+    assert st("ds_compact64_ex", FAKE, 1 << 40, 0, None, None) == UNS    # > 2^35 elements
+    assert st("ds_unique64", FAKE, 10, None) == INV                      # out_n required
+    n = ctypes.c_size_t(99)
+    assert st("ds_unique64", FAKE, 0, ctypes.byref(n)) == 0 and n.value == 0

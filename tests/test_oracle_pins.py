@@ -396,3 +396,73 @@ def test_golden_worked_examples(case):
         assert m == case["out_n"]
         assert np.array_equal(a[:m], case["output"])
     assert np.array_equal(a, case["buffer_after"])
+
+
+# ------------------------------------------------------ 8-byte elements
+def _rand64(n, seed, alphabet=None):
+    rng = np.random.default_rng(seed)
+    if alphabet is not None:
+        return rng.choice(np.array(alphabet, dtype=np.uint64), size=n).astype(np.uint64)
+    return rng.integers(0, 2**64, size=n, dtype=np.uint64)
+
+
+def test_compact64_brute_force_and_numpy_mask():
+    """All keep/remove patterns up to n = 10 (value 0 vs nonzero), then numpy
+    boolean masking on random data; the high word alone must decide too."""
+    for n in range(0, 11):
+        for mask in range(1 << n):
+            a = np.array([(i + 1) if (mask >> i) & 1 else 0 for i in range(n)], dtype=np.uint64)
+            exp = a[a != 0].copy()
+            m = oracle.compact64(a, 0)
+            assert m == exp.size and np.array_equal(a[:m], exp)
+    v = np.uint64(0xDEADBEEF00000001)
+    a = np.array([v, 1, 0xDEADBEEF00000000, v, 0x00000001DEADBEEF], dtype=np.uint64)
+    exp = a[a != v].copy()
+    m = oracle.compact64(a, int(v))
+    assert m == 3 and np.array_equal(a[:m], exp)
+    a = _rand64(50_000, 3, alphabet=[5, 7, 1 << 40, (1 << 40) + 5])
+    orig = a.copy()
+    m = oracle.compact64(a, 1 << 40)
+    exp = orig[orig != np.uint64(1 << 40)]
+    assert m == exp.size and np.array_equal(a[:m], exp) and np.array_equal(a[m:], orig[m:])
+
+
+@pytest.mark.parametrize("pred", range(oracle.PRED_COUNT))
+def test_select64_equals_numpy(pred):
+    rng = np.random.default_rng(10 + pred)
+    if pred in (3, 4):  # doubles, with NaN / -0.0 / inf patterns
+        d = rng.normal(size=20_000)
+        d[::97] = np.nan
+        d[::89] = -0.0
+        d[::83] = np.inf
+        a = d.view(np.uint64).copy()
+        param = np.array([0.25]).view(np.uint64)[0]
+        dd, pd = a.view(np.float64), np.array([0.25])[0]
+        keep = (dd > pd) if pred == 3 else ~(dd > pd)
+    else:
+        a = rng.integers(-2**62, 2**62, size=20_000, dtype=np.int64).view(np.uint64).copy()
+        a[::7] = 0
+        param = np.uint64(12345)
+        s = a.view(np.int64)
+        keep = {0: a != 0, 1: s > 12345, 2: ~(s > 12345), 5: (a & np.uint64(1)) == 0,
+                6: (a & np.uint64(1)) != 0}[pred]
+    exp = a[keep].copy()
+    m = oracle.select64(a, pred, int(param))
+    assert m == exp.size and np.array_equal(a[:m], exp)
+
+
+def test_unique64_brute_force_and_numpy():
+    """Every sequence of length <= 7 over a 2-letter alphabet that differs only
+    in the high word, then the numpy consecutive-difference mask."""
+    letters = [np.uint64(3), np.uint64(3 + (1 << 32))]
+    for n in range(0, 8):
+        for bits in itertools.product([0, 1], repeat=n):
+            a = np.array([letters[b] for b in bits], dtype=np.uint64)
+            exp = [a[i] for i in range(n) if i == 0 or a[i] != a[i - 1]]
+            m = oracle.unique64(a)
+            assert m == len(exp) and list(a[:m]) == exp
+    a = _rand64(100_000, 4, alphabet=[1, 2, 2**63])
+    orig = a.copy()
+    keep = np.concatenate([[True], orig[1:] != orig[:-1]])
+    m = oracle.unique64(a)
+    assert m == int(keep.sum()) and np.array_equal(a[:m], orig[keep])

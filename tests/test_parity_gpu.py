@@ -397,3 +397,65 @@ def test_slide_ex_stream_repeated():
         libds.ds_slide_ex(buf.ptr, n, shift, 4, s)
     s.synchronize()
     buf.assert_equals(exp, "slide repeated")
+
+
+# ------------------------------------------------------ 8-byte elements
+SIZES64 = [1, 2, 3, 16, 2047, 4096, 4097, 8191, 3 * 4096 + 5, 100_003, 1_000_003]
+
+
+def _dev64(host, mis):
+    """DevBuf over the uint64 array's words; mis in {0, 2} keeps 8-byte alignment."""
+    return DevBuf(host.view(np.uint32), mis)
+
+
+@pytest.mark.parametrize("n", SIZES64)
+@pytest.mark.parametrize("mis", [0, 2])
+def test_compact64(n, mis):
+    rng = np.random.default_rng(n + mis)
+    for f in (0.0, 0.3, 1.0):
+        vals = rng.integers(1, 2**64, size=n, dtype=np.uint64)
+        rm = np.uint64(0xABCD000000000000)
+        host = np.where(rng.random(n) < f, vals, rm).astype(np.uint64)
+        host[::11] = rm ^ np.uint64(1 << 32)  # same low word as the removed value: kept
+        buf = _dev64(host, mis)
+        exp = buf.host_region()
+        m_exp = oracle.compact64(exp.view(np.uint64), int(rm))
+        m = libds.ds_compact64(buf.ptr, n, int(rm))
+        assert m == m_exp
+        buf.assert_equals(exp, f"compact64 n={n} mis={mis} f={f}")
+
+
+@pytest.mark.parametrize("pred", range(libds.DS_PRED_COUNT))
+@pytest.mark.parametrize("n", [5, 4097, 250_001])
+def test_select64(pred, n):
+    rng = np.random.default_rng(pred * 7 + n)
+    if pred in (3, 4):
+        d = rng.normal(size=n)
+        d[::13] = np.nan
+        host = d.view(np.uint64).copy()
+        param = int(np.array([0.1]).view(np.uint64)[0])
+    else:
+        host = rng.integers(-2**62, 2**62, size=n, dtype=np.int64).view(np.uint64).copy()
+        host[::5] = 0
+        param = 1 << 40
+    buf = _dev64(host, 2)
+    exp = buf.host_region()
+    m_exp = oracle.select64(exp.view(np.uint64), pred, param)
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    libds.ds_select64_ex(buf.ptr, n, pred, param, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == m_exp
+    buf.assert_equals(exp, f"select64 pred={pred} n={n}")
+
+
+@pytest.mark.parametrize("n", SIZES64)
+def test_unique64(n):
+    rng = np.random.default_rng(3 * n)
+    letters = np.array([7, 7 + (1 << 32), 1 << 63], dtype=np.uint64)
+    runs = rng.integers(1, 5, size=n)
+    host = np.repeat(rng.choice(letters, size=n), runs)[:n].astype(np.uint64)
+    buf = _dev64(host, 0)
+    exp = buf.host_region()
+    m_exp = oracle.unique64(exp.view(np.uint64))
+    assert libds.ds_unique64(buf.ptr, n) == m_exp
+    buf.assert_equals(exp, f"unique64 n={n}")

@@ -7,6 +7,7 @@
 //   tma_copy<S,CH>:  bulk load + bulk store of the same chunk (read+write).
 // Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o bw_probe tools/bw_probe.cu
 #include <cstdio>
+#include <cstdlib>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -85,6 +86,24 @@ __global__ void ldg_kernel(const uint4* __restrict__ src, size_t n16, unsigned l
     if (acc == 0x1234567) atomicAdd(sink, acc);
 }
 
+__global__ void gtimer_kernel(unsigned long long* out) {
+    long long c0 = clock64();
+    unsigned long long g = 0, acc = 0;
+    for (int i = 0; i < 100; ++i) {
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+        acc += g;
+    }
+    long long c1 = clock64();
+    unsigned long long g0, g1;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g0));
+    long long c2 = clock64();
+    while (clock64() - c2 < 100000) {}
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g1));
+    out[0] = (c1 - c0) / 100;
+    out[1] = g1 - g0;
+    out[2] = acc;
+}
+
 __global__ void flush_kernel(uint4* p, size_t n16) {
     for (size_t i = size_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n16; i += size_t(gridDim.x) * blockDim.x)
         p[i] = make_uint4(i, 0, 0, 0);
@@ -119,6 +138,15 @@ int main() {
         CK(cudaGetLastError());
         printf("%-44s %8.1f us  %7.1f GB/s\n", name, best * 1e3, traffic / (best * 1e-3) / 1e9);
     };
+    {
+        unsigned long long h[3];
+        unsigned long long* d3;
+        CK(cudaMalloc(&d3, 24));
+        gtimer_kernel<<<1, 1>>>(d3);
+        CK(cudaMemcpy(h, d3, 24, cudaMemcpyDeviceToHost));
+        printf("globaltimer read: %llu cycles each; 100000 cycles = %llu ns of globaltimer\n", h[0], h[1]);
+        if (getenv("GT_ONLY")) return 0;
+    }
     struct Cfg { int S, CH, ctas; };
     const Cfg cfgs[] = {{6, 32768, 1}, {3, 65536, 1}, {12, 16384, 1}, {24, 8192, 1}, {6, 16384, 2}, {3, 32768, 2},
                         {12, 8192, 2}, {4, 16384, 3}, {6, 8192, 4}, {13, 16384, 1}};

@@ -6,4 +6,4 @@ timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; ech
 timeout 600 python bench.py --impl reference > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 3 --no-rows --no-e2e --no-cpu > gpurun_out/ncu_list.log 2>&1
 timeout 1200 ncu --set full --clock-control none --import-source on -k regex:irregular_kernel -s 3 -c 1 -o gpurun_out/prof_headline -f python bench.py --steps 1 --warmup 3 --no-rows --no-e2e --no-cpu > gpurun_out/ncu_full.log 2>&1
-tail -3 gpurun_out/smoke.log gpurun_out/pytest_gpu.log gpurun_out/bench.err; tail -2 gpurun_out/ncu_full.log
+tail -n 3 gpurun_out/smoke.log gpurun_out/pytest_gpu.log gpurun_out/bench.err; tail -n 2 gpurun_out/ncu_full.log

@@ -15,7 +15,7 @@ dev = torch.device("cuda")
 flush = torch.empty(256 << 20, dtype=torch.int32, device=dev)
 
 
-def timeit(name, pristine, fn, bytes_fn, reps=10):
+def timeit(name, pristine, fn, bytes_fn, reps=15):
     work = pristine.clone()
     d_n = torch.zeros(1, dtype=torch.int64, device=dev)
     ts = []

@@ -54,6 +54,11 @@ def main():
                     ("lb:fence", lb[:, 2] - lb[:, 1]), ("lb:publish", ev[:, 4] - lb[:, 2])):
         q = np.percentile(d[1:], [5, 50, 95, 99])
         print(f"{name:13s} p5 {q[0]:7.2f}  p50 {q[1]:7.2f}  p95 {q[2]:7.2f}  p99 {q[3]:7.2f}")
+    sub = (t[:, [1, 13, 14, 2]] - t0) / 1e3
+    for name, d in (("cnt:own-warp", sub[:, 1] - sub[:, 0]), ("cnt:barrier", sub[:, 2] - sub[:, 1]),
+                    ("cnt:publish", sub[:, 3] - sub[:, 2])):
+        q = np.percentile(d, [5, 50, 95, 99])
+        print(f"{name:13s} p5 {q[0]:7.2f}  p50 {q[1]:7.2f}  p95 {q[2]:7.2f}  p99 {q[3]:7.2f}")
     print("rounds p50/p99", np.percentile(t[1:, 8], [50, 99]), "polls p50/p99", np.percentile(t[1:, 9], [50, 99]))
     agg_max_lower = np.maximum.accumulate(np.concatenate([[0.0], ev[:-1, 2]]))
     ready = np.maximum(agg_max_lower, ev[:, 3])  # every lower AGG published and look-back started
