@@ -10,21 +10,25 @@
 //                    a2 loads the tile (plus, for unique, the 16 bytes before
 //                       it) with one TMA bulk copy (Alg. 2 lines 1-11; P:84
 //                       "on-chip memory")
-//  16 ranker warps   a3 keep flags (predicate / unique stencil)
-//                    a4 per-warp counts and the tile aggregate ("Reduction",
-//                       P:182) -- published as AGG at once
+//  16 ranker warps   a3 keep flags (predicate / unique stencil), one
+//                       ballot per 32-word chunk (lane l holds word 32c + l)
+//                    a4 the tile aggregate ("Reduction") -- published
+//                       as AGG at once
 //                    a6 rank of every kept word in input order ("binary
-//                       prefix sum": ballot/popc inside each
-//                       warp's contiguous 512-word segment + a scan of the 16
-//                       warp totals); the kept words are compacted in place
-//   6 resolver warps a5 (one per stage) decoupled look-back over 512
+//                       prefix sum": popc of the chunk ballot
+//                       below the lane + a scan of the 16 warp totals); the
+//                       kept words are compacted in place, 32 consecutive
+//                       words per store
+//   6 resolver warps a5 (one per stage) decoupled look-back over 128
 //                       predecessors per round trip, started as soon as the
 //                       ticket is drawn (it needs no data), then INCL; the last
 //                       tile writes out_n (a8).  This replaces the serial flag
 //                       chain of Fig. 7, which is latency-bound on B200
-//                       (DESIGN.md §5)
-//   6 storer warps   a7 128-bit stores of the compacted tile to
-//                       [excl, excl + A) (scalar head/tail), then free the stage
+//                       (DESIGN.md §4.4)
+//   5 storer warps   a7 re-phase the compacted words in shared memory to the
+//                       destination's 16-byte phase, one TMA bulk store of
+//                       [excl, excl + A) (scalar head/tail), then free the
+//                       stage once the bulk engine has read it
 //
 // A drawn tile's AGG depends only on its own load and ranking, never on the
 // resolution of earlier tiles.  In-place safety:
@@ -546,15 +550,13 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint64_t tb = uint64_t(t) * kT;
             uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
             end = (end + 3) & ~3ull;  // may read <= 12 bytes past the array end (same 16 B chunk)
-            // The tile itself from its 128-byte aligned start; unique's 16 bytes
-            // before it as a second copy (one unaligned copy would touch an extra
-            // line per request block).
-            const bool pre = Op::kUnique && t > 0;
-            const uint32_t bytes = uint32_t(end - tb) * 4u;
+            // Unique also needs the word before the tile: one copy starting 16
+            // bytes early (measured faster than a separate 16-byte copy).
+            const uint64_t beg = (Op::kUnique && t > 0) ? tb - kPre : tb;
+            const uint32_t bytes = uint32_t(end - beg) * 4u;
             fence_proxy_async_smem();
-            mbar_arrive_expect_tx(&bar_full[s], bytes + (pre ? 16u : 0u));
-            if (pre) bulk_g2s(stage, p.abase + tb - kPre, 16u, &bar_full[s]);
-            bulk_g2s(stage + kPre, p.abase + tb, bytes, &bar_full[s]);
+            mbar_arrive_expect_tx(&bar_full[s], bytes);
+            bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_full[s]);
         }
     } else if (warp < kRankWarps) {
         // ------------------------------------------------ ranker warps
