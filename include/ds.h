@@ -49,8 +49,9 @@ typedef struct CUstream_st* ds_stream_t;
 typedef enum ds_status {
     DS_SUCCESS = 0,
     DS_ERROR_INVALID_VALUE = 1, /* NULL pointer, misaligned ptr, bad sizes  */
-    DS_ERROR_UNSUPPORTED = 2,   /* valid but not implemented (elem_bytes 1/2,
-                                   n >= 2^36 words, rows longer than 2^30 words) */
+    DS_ERROR_UNSUPPORTED = 2,   /* valid but not implemented (ds_slide with
+                                   elem_bytes 1/2, n >= 2^36 words, rows longer
+                                   than 2^30 words) */
     DS_ERROR_OUT_OF_MEMORY = 3, /* workspace allocation failed              */
     DS_ERROR_CUDA = 4           /* a CUDA runtime call failed               */
 } ds_status;
@@ -81,7 +82,10 @@ typedef enum ds_predicate {
  * After the call ptr holds rows x new_cols: row i moved forward by
  * (new_cols-cols)*i elements ("row i will be shifted by C x i") and
  * followed by new_cols-cols fill elements (zero bytes, R1/R2).
- * Requires new_cols >= cols; elem_bytes in {4, 8, 16}.                   */
+ * Requires new_cols >= cols; elem_bytes in {1, 2, 4, 8, 16}.  ptr must be
+ * aligned to min(elem_bytes, 4).  1- and 2-byte elements whose rows are
+ * not whole 32-bit words run on a byte-granular variant of the same kernel
+ * (SURVEY 8(f)-4); rows longer than 2^30 words return DS_ERROR_UNSUPPORTED. */
 ds_status ds_pad(void* ptr, size_t rows, size_t cols, size_t new_cols,
                  size_t elem_bytes);
 

@@ -23,7 +23,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-SOURCES = ["ds_api.cu", "ds_irregular.cu", "ds_regular.cu", "ds_shard.cu"]
+SOURCES = ["ds_api.cu", "ds_irregular.cu", "ds_regular.cu", "ds_regular_bytes.cu", "ds_shard.cu"]
 HEADERS = ["ds_device.cuh", "ds_internal.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 VARIANTS = {

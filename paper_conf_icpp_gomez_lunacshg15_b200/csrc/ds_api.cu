@@ -132,9 +132,56 @@ ds_status irregular_blocking(ds::IrregArgs a, size_t* out_n) {
     return DS_SUCCESS;
 }
 
+ds_status run_regular(const ds::RegArgs& a, cudaStream_t s);
+
+// Sub-word elements (eb 1, 2): rows of whole words run on the word kernel
+// (the fill replicated into a word); anything else on the byte kernel.
+ds_status run_sub_word(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t eb, bool pad,
+                       const void* fill, cudaStream_t s) {
+    if (pad ? new_cols < cols : new_cols > cols) return DS_ERROR_INVALID_VALUE;
+    size_t big = pad ? new_cols : cols, tmp = 0;
+    if (__builtin_mul_overflow(rows, big, &tmp) || __builtin_mul_overflow(tmp, eb, &tmp))
+        return DS_ERROR_INVALID_VALUE;
+    if (tmp > 0 && ptr == nullptr) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(ptr, eb)) return DS_ERROR_INVALID_VALUE;
+    if (uint64_t(big) * eb >= kMaxRowWords) return DS_ERROR_UNSUPPORTED;
+    if (tmp / 4 > kMaxMatrixWords) return DS_ERROR_UNSUPPORTED;
+    uint8_t f[2] = {0, 0};
+    if (fill) std::memcpy(f, fill, eb);
+    if (eb == 1) f[1] = f[0];
+    const uint64_t cb = uint64_t(cols) * eb, ncb = uint64_t(new_cols) * eb;
+    if (rows == 0 || cb == ncb || ncb == 0) return DS_SUCCESS;  // nothing moves
+    if (cb % 4 == 0 && ncb % 4 == 0 && !misaligned(ptr, 4)) {
+        ds::RegArgs a{};
+        a.ptr = static_cast<uint32_t*>(ptr);
+        a.rows = rows;
+        a.cols_w = cb / 4;
+        a.new_cols_w = ncb / 4;
+        a.words_per_elem = 1;
+        a.pad = pad;
+        const uint32_t w = uint32_t(f[0]) | uint32_t(f[1]) << 8;
+        a.fill[0] = a.fill[1] = a.fill[2] = a.fill[3] = w | w << 16;
+        return run_regular(a, s);
+    }
+    ds::RegBytesArgs b{};
+    b.ptr = static_cast<uint8_t*>(ptr);
+    b.rows = rows;
+    b.cols_b = cb;
+    b.new_cols_b = ncb;
+    b.elem_bytes = uint32_t(eb);
+    b.fill[0] = f[0];
+    b.fill[1] = f[1];
+    b.pad = pad;
+    std::lock_guard<std::mutex> lock(g_mu);
+    ds::Workspace* ws = nullptr;
+    ds_status st = get_workspace(ds::regular_bytes_tiles(b), s, &ws);
+    if (st != DS_SUCCESS) return st;
+    cudaError_t e = ds::launch_regular_bytes(b, *ws, s);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "regular bytes kernel launch");
+}
+
 ds_status check_regular(const void* ptr, size_t rows, size_t cols, size_t new_cols, size_t eb,
                         bool pad, ds::RegArgs* a) {
-    if (eb == 1 || eb == 2) return DS_ERROR_UNSUPPORTED;
     if (eb != 4 && eb != 8 && eb != 16) return DS_ERROR_INVALID_VALUE;
     if (pad ? new_cols < cols : new_cols > cols) return DS_ERROR_INVALID_VALUE;
     size_t big = pad ? new_cols : cols, tmp = 0;
@@ -204,6 +251,9 @@ extern "C" {
 
 ds_status ds_pad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes,
                     const void* fill, ds_stream_t stream) {
+    if (elem_bytes == 1 || elem_bytes == 2)
+        return run_sub_word(ptr, rows, cols, new_cols, elem_bytes, true, fill,
+                            reinterpret_cast<cudaStream_t>(stream));
     ds::RegArgs a{};
     ds_status st = check_regular(ptr, rows, cols, new_cols, elem_bytes, true, &a);
     if (st != DS_SUCCESS) return st;
@@ -213,6 +263,9 @@ ds_status ds_pad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t
 
 ds_status ds_unpad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes,
                       ds_stream_t stream) {
+    if (elem_bytes == 1 || elem_bytes == 2)
+        return run_sub_word(ptr, rows, cols, new_cols, elem_bytes, false, nullptr,
+                            reinterpret_cast<cudaStream_t>(stream));
     ds::RegArgs a{};
     ds_status st = check_regular(ptr, rows, cols, new_cols, elem_bytes, false, &a);
     if (st != DS_SUCCESS) return st;

@@ -48,6 +48,17 @@ struct RegArgs {
     uint64_t out_words_w = 0;  // slide: output words (0: rows * new_cols_w)
 };
 
+// 1- and 2-byte elements whose rows are not whole words (ds_regular_bytes.cu).
+struct RegBytesArgs {
+    uint8_t* ptr;
+    uint64_t rows;
+    uint64_t cols_b;      // bytes per row before
+    uint64_t new_cols_b;  // bytes per row after
+    uint32_t elem_bytes;  // 1 or 2
+    uint8_t fill[2];
+    bool pad;
+};
+
 // Tiles a launch of each kernel family needs (for workspace sizing).
 size_t irregular_tiles(const IrregArgs& a);
 size_t regular_tiles(const RegArgs& a);
@@ -55,6 +66,8 @@ size_t regular_tiles(const RegArgs& a);
 // Enqueue the kernels; return the cudaError_t of the launch.
 cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s);
 cudaError_t launch_regular(const RegArgs& a, Workspace& ws, cudaStream_t s);
+size_t regular_bytes_tiles(const RegBytesArgs& a);
+cudaError_t launch_regular_bytes(const RegBytesArgs& a, Workspace& ws, cudaStream_t s);
 // Copies n words src[0, n) -> dst_base[*d_offset + j] (partition's tail move).
 cudaError_t launch_tail_copy(uint32_t* dst_base, const uint64_t* d_offset, const uint32_t* src,
                              const uint64_t* d_count_false, size_t n_total, cudaStream_t s);

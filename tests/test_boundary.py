@@ -96,8 +96,12 @@ def test_regular_validation_before_device():
     assert st("ds_unpad", FAKE, 4, 4, 5, 4) == INV        # new_cols > cols
     assert st("ds_pad", FAKE, 4, 4, 5, 3) == INV          # bad elem_bytes
     assert st("ds_pad", FAKE, 4, 4, 5, 0) == INV
-    assert st("ds_pad", FAKE, 4, 4, 5, 2) == UNS          # 1/2-byte elements: NEXT
-    assert st("ds_unpad", FAKE, 4, 5, 4, 1) == UNS
+    assert st("ds_pad", FAKE, 4, 5, 4, 2) == INV          # 2-byte elements: new_cols < cols
+    assert st("ds_unpad", FAKE, 4, 4, 5, 1) == INV        # 1-byte elements: new_cols > cols
+    assert st("ds_pad", FAKE + 1, 4, 4, 5, 2) == INV      # 2-byte elements, odd address
+    assert st("ds_pad", None, 4, 4, 5, 1) == INV
+    assert st("ds_pad", FAKE, 2, 1, 1 << 31, 1) == UNS    # row longer than 2^30 words
+    assert st("ds_pad_ex", FAKE + 3, 0, 5, 9, 1, None, None) == 0   # rows == 0: nothing to do
     assert st("ds_pad", None, 4, 4, 5, 4) == INV          # NULL with data
     assert st("ds_pad", BAD, 4, 4, 5, 4) == INV           # misaligned
     assert st("ds_pad", FAKE, 1 << 40, 1 << 30, 1 << 31, 8) == INV   # size overflow

@@ -290,6 +290,26 @@ def test_pad_unpad_brute_force_small():
                     assert np.array_equal(buf[R * C * w:], exp[R * C * w:])
 
 
+def test_pad_unpad_sub_word_elements():
+    """1- and 2-byte elements (8(f)-4): numpy.pad on the element view, the
+    round trip, for every R <= 3, C <= 6, NC <= 9."""
+    for eb, dt in ((1, np.uint8), (2, np.uint16)):
+        fill = bytes([0xA5, 0x5A][:eb])
+        fv = np.frombuffer(fill, dtype=dt)[0]
+        for R in range(0, 4):
+            for C in range(0, 7):
+                for NC in range(C, 10):
+                    buf = np.arange(R * NC * eb + 5, dtype=np.uint8) * np.uint8(37) + np.uint8(11)
+                    orig = buf.copy()
+                    oracle.pad(buf, R, C, NC, eb, fill)
+                    m = orig[:R * C * eb].view(dt).reshape(R, C)
+                    exp = np.pad(m, ((0, 0), (0, NC - C)), constant_values=fv).reshape(-1).view(np.uint8)
+                    assert np.array_equal(buf[:R * NC * eb], exp), (eb, R, C, NC)
+                    assert np.array_equal(buf[R * NC * eb:], orig[R * NC * eb:])
+                    oracle.unpad(buf, R, NC, C, eb)
+                    assert np.array_equal(buf[:R * C * eb], orig[:R * C * eb])
+
+
 def test_unpad_equals_slicing():
     R, C, NC = 37, 53, 41
     buf = dsgen.matrix_input(R, C, NC, 4).numpy().view(np.uint32).copy()

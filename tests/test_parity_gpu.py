@@ -459,3 +459,93 @@ def test_unique64(n):
     m_exp = oracle.unique64(exp.view(np.uint64))
     assert libds.ds_unique64(buf.ptr, n) == m_exp
     buf.assert_equals(exp, f"unique64 n={n}")
+
+
+# ------------------------------------------------- 1- and 2-byte elements (8(f)-4)
+class ByteBuf:
+    """Device bytes at a chosen byte offset past a 16-byte boundary, with 64
+    canary bytes on each side; compared as a whole."""
+
+    def __init__(self, host_bytes, mis):
+        self.pre = 64 + mis
+        full = np.empty(self.pre + host_bytes.size + 64, dtype=np.uint8)
+        full[:self.pre] = (np.arange(self.pre) * 7 + 3).astype(np.uint8)
+        full[self.pre:self.pre + host_bytes.size] = host_bytes
+        full[self.pre + host_bytes.size:] = (np.arange(64) * 11 + 5).astype(np.uint8)
+        self.full = full
+        self.n = host_bytes.size
+        self.t = torch.from_numpy(full.copy()).to("cuda")
+        assert self.t.data_ptr() % 16 == 0
+
+    @property
+    def ptr(self):
+        return self.t.data_ptr() + self.pre
+
+    def region(self):
+        return self.full[self.pre:self.pre + self.n].copy()
+
+    def check(self, region, what):
+        torch.cuda.synchronize()
+        got = self.t.cpu().numpy()
+        exp = self.full.copy()
+        exp[self.pre:self.pre + self.n] = region
+        if not np.array_equal(got, exp):
+            bad = np.nonzero(got != exp)[0]
+            raise AssertionError(f"{what}: {bad.size} bytes differ, first at {int(bad[0]) - self.pre}")
+
+
+def _sub_word_case(R, C, NC, eb, mis, fill):
+    rng = np.random.default_rng(R * 1000003 + C * 131 + NC + eb)
+    host = rng.integers(0, 256, size=R * NC * eb, dtype=np.uint8)
+    buf = ByteBuf(host, mis)
+    exp = buf.region()
+    oracle.pad(exp, R, C, NC, eb, fill)
+    libds.ds_pad_ex(buf.ptr, R, C, NC, eb, fill, None)
+    buf.check(exp, f"pad R={R} C={C} NC={NC} eb={eb} mis={mis}")
+    back = exp.copy()
+    oracle.unpad(back, R, NC, C, eb)
+    libds.ds_unpad(buf.ptr, R, NC, C, eb)
+    buf.check(back, f"unpad R={R} C={NC} NC={C} eb={eb} mis={mis}")
+
+
+def test_sub_word_pad_unpad_small_all():
+    for eb in (1, 2):
+        fill = bytes([0xC3, 0x3C][:eb])
+        for R in (1, 2, 3, 5):
+            for C in range(0, 7):
+                for NC in range(C, 10):
+                    _sub_word_case(R, C, NC, eb, (R + C + NC) * eb % 16, fill)
+
+
+@pytest.mark.parametrize("shape", [
+    (4000, 3990, 4000, 1),     # C2 shape in bytes (rows not whole words)
+    (4000, 3990, 4000, 2),
+    (5000, 4900, 5000, 1),
+    (777, 1023, 1025, 2),
+    (3, 1_000_001, 1_000_003, 1),
+    (100_000, 3, 5, 1),        # tiny rows: byte-wise chunks everywhere
+    (2000, 1, 5000, 1),        # huge padding: fill chunks, wide windows
+    (300, 20_000, 19_999, 2),  # unpad-style (pad from 19_999 back: see round trip)
+    (1000, 4096, 4097, 1),
+    (64, 4096, 4100, 2),       # whole words: routed to the word kernel
+])
+@pytest.mark.parametrize("mis", [0, 1, 6, 15])
+def test_sub_word_pad_unpad_shapes(shape, mis):
+    R, C, NC, eb = shape
+    if NC < C:
+        C, NC = NC, C
+    if eb == 2 and mis % 2:
+        mis -= 1
+    _sub_word_case(R, C, NC, eb, mis, bytes([0x81, 0x18][:eb]))
+
+
+def test_sub_word_unpad_large_drop_slow_path():
+    """Short rows dropping many bytes: the source span exceeds a stage, so the
+    producer gathers byte by byte from global memory."""
+    for (R, C, NC, eb) in ((20_000, 5000, 3, 1), (3000, 20_001, 7, 2)):
+        host = np.random.default_rng(R).integers(0, 256, size=R * C * eb, dtype=np.uint8)
+        buf = ByteBuf(host, 3 if eb == 1 else 2)
+        exp = buf.region()
+        oracle.unpad(exp, R, C, NC, eb)
+        libds.ds_unpad(buf.ptr, R, C, NC, eb)
+        buf.check(exp, f"unpad slow R={R} C={C} NC={NC} eb={eb}")

@@ -59,6 +59,12 @@ def main():
     libds.ds_pad(b, R, C, NC, 4)
     timeit("unpad 4000x4000->3990", b, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, 4, None),
            lambda m: 4 * (2 * R * C))
+    for eb in (1, 2):
+        a = torch.randint(0, 256, (R * NC * eb,), dtype=torch.uint8, device=dev)
+        timeit(f"pad {R}x{C}->{NC} eb={eb}", a, lambda w, d, eb=eb: libds.ds_pad_ex(w, R, C, NC, eb, None, None),
+               lambda m, eb=eb: eb * (R * C + R * NC))
+        timeit(f"unpad {R}x{NC}->{C} eb={eb}", a, lambda w, d, eb=eb: libds.ds_unpad_ex(w, R, NC, C, eb, None),
+               lambda m, eb=eb: eb * (2 * R * C))
     R, C, NC = 12000, 11999, 12000
     a = dsgen.matrix_input(R, C, NC, 4, device=dev)
     timeit("pad 12000x11999->12000", a, lambda w, d: libds.ds_pad_ex(w, R, C, NC, 4, None, None),
