@@ -171,6 +171,22 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "memory");
     return;
 #endif
+#ifdef DS_MBAR_BACKOFF
+    // Polls with a growing sleep in between (no suspend hint): fewer mbarrier
+    // unit operations per wait while the TMA completes transactions on it.
+    for (uint32_t ns = 32;; ns = ns < DS_MBAR_BACKOFF ? 2 * ns : ns) {
+        uint32_t done;
+        asm volatile(
+            "{\n.reg .pred P;\n"
+            "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n"
+            "selp.u32 %0, 1, 0, P;\n}\n"
+            : "=r"(done)
+            : "r"(smem_addr(bar)), "r"(parity)
+            : "memory");
+        if (done) return;
+        __nanosleep(ns);
+    }
+#endif
     asm volatile(
         "{\n"
         ".reg .pred P;\n"

@@ -132,15 +132,29 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 #ifndef DS_IRR_RESOLVERS
 #define DS_IRR_RESOLVERS 6
 #endif
+#ifndef DS_IRR_RANK_GROUPS
+#define DS_IRR_RANK_GROUPS 1
+#endif
+#ifndef DS_IRR_TILE
+#define DS_IRR_TILE 8192
+#endif
 constexpr int kRankWarps = DS_IRR_RANK_WARPS;
-constexpr int kRT = 32 * kRankWarps;      // ranker threads
-constexpr int kSeg = 512;                 // contiguous words ranked by one warp
-constexpr int kChunks = kSeg / 32;        // 32-word chunks per warp segment (16)
-constexpr int kT = kRankWarps * kSeg;     // words per tile (8192 = 32 KB with 16 rankers)
+constexpr int kRankGroups = DS_IRR_RANK_GROUPS;   // ranker groups, each on its own tile
+constexpr int kGroupWarps = kRankWarps / kRankGroups;
+constexpr int kRT = 32 * kGroupWarps;     // threads of one ranker group
+constexpr int kT = DS_IRR_TILE;           // words per tile (8192 = 32 KB)
+constexpr int kSeg = kT / kGroupWarps;    // contiguous words ranked by one warp (1024)
+constexpr int kChunks = kSeg / 32;        // 32-word chunks per warp segment (32)
+static_assert(kRankWarps % kRankGroups == 0 && kT % (32 * kGroupWarps) == 0, "ranker shape");
+static_assert(kChunks <= 32, "chunk masks are held one per lane");
+static_assert(kRankGroups <= 2, "named barriers 1 and 3 serve the ranker groups");
 constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
 constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
 constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
-constexpr int kStoreWarps = 5;
+#ifndef DS_IRR_STORE_WARPS
+#define DS_IRR_STORE_WARPS 5
+#endif
+constexpr int kStoreWarps = DS_IRR_STORE_WARPS;
 #ifndef DS_IRR_BULK_STORE
 #define DS_IRR_BULK_STORE 1
 #endif
@@ -150,14 +164,27 @@ constexpr int kWarpResolver0 = kRankWarps;
 constexpr int kWarpStorer0 = kRankWarps + kResolvers;
 constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;
 constexpr int kThreads = 32 * (kWarpProducer + 1);
-constexpr int kPre = 4;                   // words before the tile (unique's boundary word)
-constexpr int kStageWords = kT + kPre + 4;
-constexpr size_t kSmem = size_t(kInStages) * kStageWords * 4;
-static_assert(kRankWarps <= 32, "warp-total scan in one warp");
+#ifndef DS_IRR_PRE
+#define DS_IRR_PRE 32
+#endif
+// Words before the tile in a stage (unique's boundary word).  Stages, and the
+// tile inside each stage, start on 128-byte boundaries, so a bulk copy fills
+// whole 128-byte shared-memory lines and unique's copy (which starts kPre
+// words early) keeps a 128-byte aligned global source.
+constexpr int kPre = DS_IRR_PRE;
+#ifndef DS_IRR_ALIGN
+#define DS_IRR_ALIGN 32
+#endif
+constexpr int kAlignW = DS_IRR_ALIGN;    // stage alignment in words (32 = 128 bytes)
+constexpr int kStageWords = (kT + kPre + 4 + kAlignW - 1) / kAlignW * kAlignW;
+constexpr size_t kSmem = size_t(kInStages) * kStageWords * 4 + 128;  // + runtime alignment slack
+static_assert(kPre % 4 == 0 && kPre >= 4, "boundary words keep 16-byte alignment");
 static_assert(kThreads <= 1024, "CTA size");
 static_assert(kSlots >= kInStages, "a slot per input stage at least");
 static_assert(kSlots % kResolvers == 0, "a slot is always served by the same resolver");
-static_assert(kSmem <= 227 * 1024 - 4096, "shared memory");
+// 227 KB dynamic + static per CTA (the static part -- barriers, slot metadata --
+// is < 2.5 KB)
+static_assert(kSmem <= 227 * 1024 - 2560, "shared memory");
 
 struct SlotMeta {
     uint32_t tile;              // kNoTile: end of this CTA's work
@@ -166,7 +193,7 @@ struct SlotMeta {
     volatile unsigned long long incl;     // inclusive prefix of the tile
     uint32_t total;             // kept words in the tile
     unsigned long long excl;    // kept words in all lower tiles
-    uint32_t wtot[kRankWarps];  // kept words in each ranker warp's segment
+    uint32_t wtot[kGroupWarps];  // kept words in each ranker warp's segment
 };
 
 // Shard halo (R18): last word of the nearest non-empty earlier shard.
@@ -203,6 +230,16 @@ constexpr int kRefreshRows = DS_IRR_REFRESH;        // AGG rows re-read while po
 constexpr uint32_t kPollMinNs = DS_IRR_POLL_MIN;   // first back-off
 constexpr uint32_t kPollMaxNs = DS_IRR_POLL_MAX;   // back-off cap
 
+// Timing experiments only (wrong or unsafe results): DS_DEBUG_BISECT bits
+#ifndef DS_DEBUG_BISECT
+#define DS_DEBUG_BISECT 0
+#endif
+constexpr bool DBG_NO_PFENCE = DS_DEBUG_BISECT & 1, DBG_NO_PUBLISH = DS_DEBUG_BISECT & 2,
+               DBG_NO_BULKWAIT = DS_DEBUG_BISECT & 4, DBG_EARLY_FREE = DS_DEBUG_BISECT & 8,
+               DBG_SKIP_RANK = DS_DEBUG_BISECT & 16, DBG_NO_RFENCE = DS_DEBUG_BISECT & 32;
+#ifndef DS_IRR_LATE_LB
+#define DS_IRR_LATE_LB 0
+#endif
 #ifndef DS_IRR_HELP
 #define DS_IRR_HELP 0
 #endif
@@ -495,7 +532,10 @@ __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
 
 template <class Op, bool PART>
 __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParams p) {
-    extern __shared__ __align__(128) uint32_t smem[];
+    extern __shared__ __align__(128) uint32_t smem_raw[];
+    // 128-byte aligned stage base (offset arithmetic keeps the shared window,
+    // so the stage accesses stay LDS/STS)
+    uint32_t* const smem = smem_raw + ((128u - (smem_addr(smem_raw) & 127u)) & 127u) / 4u;
     __shared__ __align__(8) uint64_t bar_full[kInStages], bar_free[kInStages];
     __shared__ __align__(8) uint64_t bar_drawn[kSlots], bar_counted[kSlots], bar_ranked[kSlots],
         bar_resolved[kSlots], bar_stored[kSlots];
@@ -512,7 +552,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         for (int o = 0; o < kSlots; ++o) {
             mbar_init(&bar_drawn[o], 1);
             mbar_init(&bar_counted[o], 1);
-            mbar_init(&bar_ranked[o], kRankWarps);
+            mbar_init(&bar_ranked[o], kGroupWarps);
             mbar_init(&bar_resolved[o], 1);
             mbar_init(&bar_stored[o], 1);
         }
@@ -554,34 +594,55 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             // bytes early (measured faster than a separate 16-byte copy).
             const uint64_t beg = (Op::kUnique && t > 0) ? tb - kPre : tb;
             const uint32_t bytes = uint32_t(end - beg) * 4u;
-            fence_proxy_async_smem();
+            if (!DBG_NO_PFENCE) fence_proxy_async_smem();
             mbar_arrive_expect_tx(&bar_full[s], bytes);
             bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_full[s]);
         }
     } else if (warp < kRankWarps) {
         // ------------------------------------------------ ranker warps
-        const int rw = warp, rt = tid;
+        // kRankGroups groups of kGroupWarps warps; group g ranks the tiles at
+        // ring positions k = g (mod kRankGroups), so one group's barrier, scan
+        // and status store overlap the other group's loads and ballots.
+        const int g = warp / kGroupWarps, rw = warp % kGroupWarps;
+        const int rt = tid - g * kRT;  // thread index within the group
+        const uint32_t gbar = 1 + 2 * g;  // named barrier of the group (2 is the storers')
         const uint32_t lt = lanemask_lt();
         bool has_hprev = false;
         uint32_t hprev = 0;
         if (Op::kUnique) has_hprev = halo_prev(p, hprev);
-        for (uint32_t k = 0;; ++k) {
+        for (uint32_t k = g;; k += kRankGroups) {
             const int s = k % kInStages, o = k % kSlots;
             uint32_t* stage = smem + s * kStageWords;
-            mbar_wait(&bar_full[s], (k / kInStages) & 1);
+            // the other group's end position releases this group too
+            if (!mbar_wait_or_end(&bar_full[s], (k / kInStages) & 1, &s_end, k)) break;
             const uint32_t t = meta[o].tile;
             if (t == kNoTile) break;
             if (rt == 0) trace_event(p.trace, t, 1, globaltimer());
+            if (DBG_SKIP_RANK) {  // timing experiment only
+                named_bar_sync(gbar, kRT);
+                if (rt == 0) {
+                    meta[o].total = 0;
+                    publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, 0));
+                    mbar_arrive(&bar_counted[o]);
+                }
+                if (lane == 0) mbar_arrive(&bar_ranked[o]);
+                continue;
+            }
             const uint64_t tb = uint64_t(t) * kT;
             const bool full = tb >= p.lo && tb + kT <= p.hi;
 
             // a3/a4: warp rw ranks tile words [xs, xs + kSeg) in kChunks chunks of
             // 32: lane l holds word x = xs + 32c + l of chunk c, so every shared
             // load and every compaction store below touches 32 consecutive words
-            // (no bank conflicts), and a chunk's keep flags are one ballot.
+            // (no bank conflicts), and a chunk's keep flags are one ballot.  The
+            // ballot of chunk c is kept by lane c (one register instead of kChunks).
             const int xs = kSeg * rw;
-            uint32_t v[kChunks], mk[kChunks];
-            uint32_t wrun = 0;  // kept words of the warp's segment
+            constexpr bool kMaskRegs = kChunks <= 16;  // else chunk c's mask is held by lane c
+            constexpr bool kRc = kMaskRegs && !PART && !Op::kUnique;  // chunk offsets from the count (registers)
+            uint32_t v[kChunks];
+            uint32_t mkr[kMaskRegs ? kChunks : 1], rc[kRc ? kChunks : 1];
+            uint32_t mymask = 0;  // lane c: keep mask of chunk c (!kMaskRegs)
+            uint32_t wrun = 0;    // kept words of the warp's segment
 #pragma unroll
             for (int c = 0; c < kChunks; ++c) v[c] = stage[kPre + xs + 32 * c + lane];
 #pragma unroll
@@ -611,31 +672,38 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                     const uint64_t e = tb + x;
                     kp = kp && e >= p.lo && e < p.hi;
                 }
-                mk[c] = __ballot_sync(kFull, kp);
-                wrun += __popc(mk[c]);
+                const uint32_t mk = __ballot_sync(kFull, kp);
+                if constexpr (kMaskRegs) {
+                    mkr[c] = mk;
+                    if constexpr (kRc) rc[c] = wrun;  // kept words of the segment before chunk c
+                } else if (lane == c) {
+                    mymask = mk;
+                }
+                wrun += __popc(mk);
             }
             if (lane == 0) meta[o].wtot[rw] = wrun;
             if (rt == 0) trace_event(p.trace, t, 13, globaltimer());
-            named_bar_sync(1, kRT);  // warp totals written; every ranker holds its words
+            named_bar_sync(gbar, kRT);  // warp totals written; every ranker holds its words
+            if (DBG_EARLY_FREE && rt == 0) mbar_arrive(&bar_free[s]);  // timing experiment only
             if (rt == 0) trace_event(p.trace, t, 14, globaltimer());
 
-            // Exclusive scan of the kRankWarps warp totals (input order), redundantly
+            // Exclusive scan of the group's warp totals (input order), redundantly
             // in every warp.
-            const uint32_t cw = lane < kRankWarps ? meta[o].wtot[lane] : 0u;
+            const uint32_t cw = lane < kGroupWarps ? meta[o].wtot[lane] : 0u;
             uint32_t iw = cw;
 #pragma unroll
-            for (int sh = 1; sh < 32; sh <<= 1) {
+            for (int sh = 1; sh < kGroupWarps; sh <<= 1) {
                 const uint32_t y = __shfl_up_sync(kFull, iw, sh);
                 if (lane >= sh) iw += y;
             }
-            const uint32_t total = __shfl_sync(kFull, iw, 31);
+            const uint32_t total = __shfl_sync(kFull, iw, kGroupWarps - 1);
             const uint32_t wbase = __shfl_sync(kFull, iw - cw, rw);
             if (rt == 0) {
                 // a4: publish the aggregate right away -- it depends on nothing else
                 // (a relaxed status store).
                 meta[o].total = total;
                 debug_delay(t, 1);
-                publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
+                if (!DBG_NO_PUBLISH) publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
                 trace_event(p.trace, t, 2, globaltimer());
                 mbar_arrive(&bar_counted[o]);
             }
@@ -650,19 +718,22 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             uint32_t r = wbase;
 #pragma unroll
             for (int c = 0; c < kChunks; ++c) {
-                const uint32_t rl = r + __popc(mk[c] & lt);  // trues before this word in the tile
-                if (mk[c] >> lane & 1u) {
+                const uint32_t mk = kMaskRegs ? mkr[c] : __shfl_sync(kFull, mymask, c);
+                if constexpr (kRc) r = wbase + rc[c];
+                const uint32_t rl = r + __popc(mk & lt);  // trues before this word in the tile
+                if (mk >> lane & 1u) {
                     out[rl] = v[c];
                 } else if (PART) {
                     const uint32_t x = uint32_t(xs + 32 * c + lane);
                     const uint64_t e = tb + x;
                     if (e >= p.lo && e < p.hi) out[total + (x - vstart) - rl] = v[c];
                 }
-                r += __popc(mk[c]);
+                if constexpr (!kRc) r += __popc(mk);
             }
-            fence_proxy_async_smem();  // the compacted words leave through a bulk store
+            if (!DBG_NO_RFENCE) fence_proxy_async_smem();  // the compacted words leave through a bulk store
             __syncwarp();
             if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is compacted
+            if (rt == 0) trace_event(p.trace, t, 15, globaltimer());
         }
     } else if (warp < kWarpStorer0) {
         // ------------------------------------------------ resolver warps
@@ -688,6 +759,9 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint64_t excl = uint64_t(t) * (kT / 2);
 #else
             uint64_t excl = 0;
+#if DS_IRR_LATE_LB  // experiment: start the look-back once the tile's own aggregate is out
+            mbar_wait(&bar_counted[o], use & 1);
+#endif
             if (t > 0) {
                 const uint32_t tp = meta[o].prev_tile;
                 if (kLocalChain && tp != kNoTile && t - tp - 1 <= uint32_t(32 * kLW))
@@ -702,7 +776,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 meta[o].incl = excl + total;  // the CTA's next tile chains on this
                 __threadfence_block();
                 meta[o].incl_tile = t;
-                if (t > 0) publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
+                if (t > 0 && !DBG_NO_PUBLISH) publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
             }
             mbar_wait(&bar_ranked[o], use & 1);  // the compacted tile is in its stage
             if (lane == 0) {
@@ -769,9 +843,9 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             named_bar_sync(2, kST);  // every storer is done reading the stage
             if (st == 0) {
                 trace_event(p.trace, t, 6, globaltimer());
-                bulk_commit();        // (possibly empty) group of this tile
-                bulk_wait_read<0>();  // the bulk engine has read the stage
-                mbar_arrive(&bar_free[s_in]);
+                if (!DBG_NO_BULKWAIT) bulk_commit();        // (possibly empty) group of this tile
+                if (!DBG_NO_BULKWAIT) bulk_wait_read<0>();  // the bulk engine has read the stage
+                if (!DBG_EARLY_FREE) mbar_arrive(&bar_free[s_in]);
                 mbar_arrive(&bar_stored[o]);
             }
         }

@@ -68,6 +68,66 @@ __global__ void __launch_bounds__(256) tma_kernel(const char* src, char* dst, si
     }
 }
 
+
+// Closer to the DS irregular kernel: optional L2 evict_first policy on the
+// loads (POL), dynamic chunk ids from a global atomic ticket (TICKET), and 16
+// "ranker" warps that each read a 512-word segment of the stage from shared
+// memory and meet at a named barrier before the stage is released (RANK).
+template <int POL, int TICKET, int RANK>
+__global__ void __launch_bounds__(1024) tma2_kernel(const char* src, size_t nchunks, int S, int CH,
+                                                   unsigned long long* ctr, unsigned long long* sink) {
+    extern __shared__ __align__(128) char sm[];
+    __shared__ __align__(8) uint64_t full[32], empty[32];
+    __shared__ uint32_t chunk_of[32];
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    if (tid == 0) {
+        for (int s = 0; s < S; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    const int nr = RANK ? 16 : 1;
+    if (warp == 0) {
+        if (tid != 0) return;
+        size_t c = blockIdx.x;
+        for (uint32_t k = 0;; ++k) {
+            const int s = k % S;
+            mbar_wait(&empty[s], ((k / S) & 1) ^ 1);
+            if (TICKET) c = atomicAdd(ctr, 1ull);
+            chunk_of[s] = c < nchunks ? uint32_t(c) : 0xffffffffu;
+            if (c >= nchunks) { mbar_arrive(&full[s]); return; }
+            mbar_expect(&full[s], CH);
+            if (POL) {
+                asm volatile("{\n.reg .b64 pol;\ncreatepolicy.fractional.L2::evict_first.b64 pol, 1.0;\n"
+                             "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], pol;\n}\n"
+                             ::"r"(sa(sm + size_t(s) * CH)), "l"(src + c * CH), "r"(CH), "r"(sa(&full[s])) : "memory");
+            } else {
+                g2s(sm + size_t(s) * CH, src + c * CH, CH, &full[s]);
+            }
+            if (!TICKET) c += gridDim.x;
+        }
+    } else if (warp <= nr) {
+        const int rw = warp - 1;
+        unsigned long long acc = 0;
+        for (uint32_t k = 0;; ++k) {
+            const int s = k % S;
+            mbar_wait(&full[s], (k / S) & 1);
+            if (chunk_of[s] == 0xffffffffu) break;
+            const uint32_t* st = reinterpret_cast<const uint32_t*>(sm + size_t(s) * CH);
+            if (RANK) {
+                const int words = CH / 4 / 16;
+                uint32_t cnt = 0;
+                for (int i = lane; i < words; i += 32) cnt += __popc(__ballot_sync(0xffffffffu, st[rw * words + i] != 0));
+                acc += cnt;
+                asm volatile("bar.sync 1, %0;" ::"r"(16 * 32) : "memory");
+                if (tid == 32) mbar_arrive(&empty[s]);
+            } else {
+                if (lane == 0) { acc += st[0]; mbar_arrive(&empty[s]); }
+            }
+        }
+        if (acc == 0x1234567) atomicAdd(sink, acc);
+    }
+}
+
 template <int U>
 __global__ void ldg_kernel(const uint4* __restrict__ src, size_t n16, unsigned long long* sink) {
     uint32_t acc = 0;
@@ -146,6 +206,25 @@ int main() {
         CK(cudaMemcpy(h, d3, 24, cudaMemcpyDeviceToHost));
         printf("globaltimer read: %llu cycles each; 100000 cycles = %llu ns of globaltimer\n", h[0], h[1]);
         if (getenv("GT_ONLY")) return 0;
+    }
+
+    if (getenv("DS_LIKE")) {
+        unsigned long long* ctr;
+        CK(cudaMalloc(&ctr, 8));
+        const int S = 6, CH = 32768;
+        const size_t smem = size_t(S) * CH, nch = bytes / CH;
+#define RUN2(P, T, R)                                                                                       \
+        {                                                                                                  \
+            CK(cudaFuncSetAttribute(tma2_kernel<P, T, R>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem))); \
+            char name[96];                                                                                 \
+            snprintf(name, sizeof name, "tma2 pol=%d ticket=%d rank=%d S=6 CH=32K", P, T, R);              \
+            timeit(name, double(bytes), [&] {                                                              \
+                cudaMemsetAsync(ctr, 0, 8);                                                                \
+                tma2_kernel<P, T, R><<<sms, R ? 32 * 17 : 64, smem>>>(a, nch, S, CH, ctr, sink);           \
+            });                                                                                            \
+        }
+        RUN2(0, 0, 0) RUN2(1, 0, 0) RUN2(0, 1, 0) RUN2(0, 0, 1) RUN2(1, 1, 1) RUN2(0, 1, 1)
+        return 0;
     }
     struct Cfg { int S, CH, ctas; };
     const Cfg cfgs[] = {{6, 32768, 1}, {3, 65536, 1}, {12, 16384, 1}, {24, 8192, 1}, {6, 16384, 2}, {3, 32768, 2},

@@ -1,0 +1,365 @@
+// rank_bench.cu -- development probe (not part of libds): cost of the irregular
+// kernel's ranking step (a3, a4, a6) in isolation, in SM cycles per 32 KB tile.
+// One CTA per SM ranks a shared-memory tile over and over (data refreshed from
+// a pristine copy each round, outside the timed part), 16 ranker warps, f = 0.5.
+//   V0: the libds ranker (lane l holds word 32c + l, one ballot per chunk,
+//       masks in registers, shuffle scan of the warp totals, in-place STS)
+//   V1: V0 with a broadcast-load scan of the warp totals
+//   V2: V1 without the compaction stores (ranking only)
+//   V3: V1 with 64-bit loads (lane l holds words 64c + 2l, +1: two ballots)
+// Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -o tools/rank_bench tools/rank_bench.cu
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <cuda_runtime.h>
+
+#define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) { printf("%s:%d %s\n", __FILE__, __LINE__, cudaGetErrorString(e_)); exit(1); } } while (0)
+
+constexpr int kW = 16, kT = 8192, kSeg = kT / kW, kChunks = kSeg / 32;
+constexpr unsigned kFull = 0xffffffffu;
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+    uint32_t m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+template <int VV>
+__global__ void __launch_bounds__(kW * 32, 1) rank_kernel(const uint32_t* src, int rounds, unsigned long long* cyc,
+                                                          unsigned long long* sink, uint32_t* dump) {
+    __shared__ __align__(128) uint32_t stage[kT + 64];
+    __shared__ uint32_t wtot[kW];
+    __shared__ __align__(16) uint32_t cexs[kW][kChunks];
+    const int tid = threadIdx.x, lane = tid & 31, rw = tid >> 5;
+    constexpr int V = VV & 15;
+    const uint32_t lt = lanemask_lt();
+    unsigned long long total_cyc = 0, acc = 0, seg_a = 0, seg_b = 0;
+    for (int it = 0; it < rounds; ++it) {
+        for (int i = tid; i < kT; i += kW * 32) stage[i] = src[(size_t(blockIdx.x) * 7 + it) % 64 * kT + i];
+        __syncthreads();
+        // BAR.SYNC blocks lazily: consume a shared word first so the timer starts
+        // after the fill (and its global loads) has really completed
+        acc += *reinterpret_cast<volatile uint32_t*>(&stage[tid]);
+        __syncthreads();
+        acc += *reinterpret_cast<volatile uint32_t*>(&stage[(tid + 1) % kT]);
+        const long long c0 = clock64();
+        const int xs = kSeg * rw;
+        uint32_t total, wbase, wrun = 0;
+        if constexpr (V == 10) {
+            // V10: no ballots, no POPC.  Lane l packs its 16 keep bits into 5-bit
+            // fields (chunk c -> register c / 6, bits 5 (c % 6)); a shuffle scan over
+            // the lanes of the packed words gives every lane, for all 16 chunks at
+            // once, the number of kept words in lower lanes (<= 31: no carries).
+            uint32_t v[kChunks];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) v[c] = stage[xs + 32 * c + lane];
+            uint32_t kb = 0, P0 = 0, P1 = 0, P2 = 0;
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                const uint32_t kp = v[c] != 0u;
+                kb |= kp << c;
+                if (c < 6) P0 |= kp << (5 * c);
+                else if (c < 12) P1 |= kp << (5 * (c - 6));
+                else P2 |= kp << (5 * (c - 12));
+            }
+            uint32_t E0 = __shfl_up_sync(kFull, P0, 1), E1 = __shfl_up_sync(kFull, P1, 1), E2 = __shfl_up_sync(kFull, P2, 1);
+            if (lane == 0) E0 = E1 = E2 = 0;
+#pragma unroll
+            for (int sh = 1; sh < 32; sh <<= 1) {
+                const uint32_t t0 = __shfl_up_sync(kFull, E0, sh), t1 = __shfl_up_sync(kFull, E1, sh),
+                               t2 = __shfl_up_sync(kFull, E2, sh);
+                if (lane >= sh) { E0 += t0; E1 += t1; E2 += t2; }
+            }
+            // chunk totals from lane 31 (exclusive count + its own bit)
+            const uint32_t L0 = __shfl_sync(kFull, E0, 31), L1 = __shfl_sync(kFull, E1, 31),
+                           L2 = __shfl_sync(kFull, E2, 31), Lk = __shfl_sync(kFull, kb, 31);
+            uint32_t rc[kChunks];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                const uint32_t Lc = c < 6 ? L0 >> (5 * c) : c < 12 ? L1 >> (5 * (c - 6)) : L2 >> (5 * (c - 12));
+                rc[c] = wrun;
+                wrun += (Lc & 31u) + (Lk >> c & 1u);
+            }
+            if (lane == 0) wtot[rw] = wrun;
+            const long long ca = clock64();
+            seg_a += ca - c0;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            const uint32_t cw = lane < kW ? wtot[lane] : 0u;
+            uint32_t iw = cw;
+#pragma unroll
+            for (int sh = 1; sh < kW; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, iw, sh);
+                if (lane >= sh) iw += y;
+            }
+            total = __shfl_sync(kFull, iw, kW - 1);
+            wbase = __shfl_sync(kFull, iw - cw, rw);
+            seg_b += clock64() - c0 + (total & 1);
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                const uint32_t Ec = c < 6 ? E0 >> (5 * c) : c < 12 ? E1 >> (5 * (c - 6)) : E2 >> (5 * (c - 12));
+                const uint32_t rl = wbase + rc[c] + (Ec & 31u);
+                if (kb >> c & 1u) stage[rl] = v[c];
+            }
+        } else if constexpr (V == 9) {
+            // V9: V0 with the chunk offsets taken from the phase-1 running count
+            uint32_t v[kChunks], mk[kChunks], rc[kChunks];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) v[c] = stage[xs + 32 * c + lane];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                mk[c] = __ballot_sync(kFull, v[c] != 0u);
+                rc[c] = wrun;
+                wrun += __popc(mk[c]);
+            }
+            if (lane == 0) wtot[rw] = wrun;
+            const long long ca = clock64();
+            seg_a += ca - c0;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            const uint32_t cw = lane < kW ? wtot[lane] : 0u;
+            uint32_t iw = cw;
+#pragma unroll
+            for (int sh = 1; sh < kW; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, iw, sh);
+                if (lane >= sh) iw += y;
+            }
+            total = __shfl_sync(kFull, iw, kW - 1);
+            wbase = __shfl_sync(kFull, iw - cw, rw);
+            seg_b += clock64() - c0 + (total & 1);
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                const uint32_t rl = wbase + rc[c] + __popc(mk[c] & lt);
+                if (mk[c] >> lane & 1u) stage[rl] = v[c];
+            }
+        } else if constexpr (V == 7 || V == 8) {
+            // V7/V8: one ballot per chunk, but no per-chunk POPC for the counts:
+            // lane c keeps chunk c's mask, one POPC + a 16-lane scan gives the
+            // chunk offsets (V7: through shared memory, V8: one shuffle per chunk)
+            uint32_t v[kChunks], mk[kChunks];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) v[c] = stage[xs + 32 * c + lane];
+            uint32_t mym = 0;
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                mk[c] = __ballot_sync(kFull, v[c] != 0u);
+                mym = lane == c ? mk[c] : mym;
+            }
+            const uint32_t cc = __popc(mym);
+            uint32_t inc = cc;
+#pragma unroll
+            for (int sh = 1; sh < kChunks; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, inc, sh);
+                if (lane >= sh) inc += y;
+            }
+            wrun = __shfl_sync(kFull, inc, kChunks - 1);
+            const uint32_t cex = inc - cc;
+            if (V == 7 && lane < kChunks) cexs[rw][lane] = cex;
+            if (lane == 0) wtot[rw] = wrun;
+            const long long ca = clock64();
+            seg_a += ca - c0;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            const uint32_t cw = lane < kW ? wtot[lane] : 0u;
+            uint32_t iw = cw;
+#pragma unroll
+            for (int sh = 1; sh < kW; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, iw, sh);
+                if (lane >= sh) iw += y;
+            }
+            total = __shfl_sync(kFull, iw, kW - 1);
+            wbase = __shfl_sync(kFull, iw - cw, rw);
+            seg_b += clock64() - c0 + (total & 1);
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                const uint32_t off = V == 7 ? cexs[rw][c] : __shfl_sync(kFull, cex, c);
+                const uint32_t rl = wbase + off + __popc(mk[c] & lt);
+                if (mk[c] >> lane & 1u) stage[rl] = v[c];
+            }
+        } else if constexpr (V == 5 || V == 6) {
+            // V5: loads + per-lane flag count + one warp reduce (no ballots)
+            // V6: loads only (xor of the words)
+            uint32_t v[kChunks];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) v[c] = stage[xs + 32 * c + lane];
+            uint32_t cnt = 0;
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) cnt += V == 5 ? uint32_t(v[c] != 0u) : v[c];
+            wrun = V == 5 ? __reduce_add_sync(kFull, cnt) : cnt;
+            if (lane == 0) wtot[rw] = wrun;
+            const long long ca = clock64();
+            seg_a += ca - c0;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            total = wtot[(rw + 1) % kW];
+            wbase = 0;
+        } else if constexpr (V == 4) {
+            constexpr int kC4 = kSeg / 128;
+            uint4 v[kC4];
+            uint32_t b[kC4][4];
+#pragma unroll
+            for (int c = 0; c < kC4; ++c) v[c] = *reinterpret_cast<const uint4*>(&stage[xs + 128 * c + 4 * lane]);
+#pragma unroll
+            for (int c = 0; c < kC4; ++c) {
+                b[c][0] = __ballot_sync(kFull, v[c].x != 0u);
+                b[c][1] = __ballot_sync(kFull, v[c].y != 0u);
+                b[c][2] = __ballot_sync(kFull, v[c].z != 0u);
+                b[c][3] = __ballot_sync(kFull, v[c].w != 0u);
+                wrun += __popc(b[c][0]) + __popc(b[c][1]) + __popc(b[c][2]) + __popc(b[c][3]);
+            }
+            if (lane == 0) wtot[rw] = wrun;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            total = 0; wbase = 0;
+#pragma unroll
+            for (int i = 0; i < kW; ++i) { const uint32_t cw = wtot[i]; wbase += i < rw ? cw : 0u; total += cw; }
+            uint32_t r = wbase;
+#pragma unroll
+            for (int c = 0; c < kC4; ++c) {
+                uint32_t q = r + __popc(b[c][0] & lt) + __popc(b[c][1] & lt) + __popc(b[c][2] & lt) + __popc(b[c][3] & lt);
+                const uint32_t w4[4] = {v[c].x, v[c].y, v[c].z, v[c].w};
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    if (b[c][j] >> lane & 1u) stage[q++] = w4[j];
+                r += __popc(b[c][0]) + __popc(b[c][1]) + __popc(b[c][2]) + __popc(b[c][3]);
+            }
+        } else if constexpr (V == 3) {
+            constexpr int kC2 = kSeg / 64;
+            uint2 v[kC2];
+            uint32_t me[kC2], mo[kC2];
+#pragma unroll
+            for (int c = 0; c < kC2; ++c) v[c] = *reinterpret_cast<const uint2*>(&stage[xs + 64 * c + 2 * lane]);
+#pragma unroll
+            for (int c = 0; c < kC2; ++c) {
+                me[c] = __ballot_sync(kFull, v[c].x != 0u);
+                mo[c] = __ballot_sync(kFull, v[c].y != 0u);
+                wrun += __popc(me[c]) + __popc(mo[c]);
+            }
+            if (lane == 0) wtot[rw] = wrun;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            total = 0; wbase = 0;
+#pragma unroll
+            for (int i = 0; i < kW; ++i) { const uint32_t cw = wtot[i]; wbase += i < rw ? cw : 0u; total += cw; }
+            uint32_t r = wbase;
+#pragma unroll
+            for (int c = 0; c < kC2; ++c) {
+                const uint32_t re = r + __popc(me[c] & lt) + __popc(mo[c] & lt);
+                const bool ke = me[c] >> lane & 1u, ko = mo[c] >> lane & 1u;
+                if (ke) stage[re] = v[c].x;
+                if (ko) stage[re + ke] = v[c].y;
+                r += __popc(me[c]) + __popc(mo[c]);
+            }
+        } else {
+            uint32_t v[kChunks], mk[kChunks];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) v[c] = stage[xs + 32 * c + lane];
+#pragma unroll
+            for (int c = 0; c < kChunks; ++c) {
+                mk[c] = __ballot_sync(kFull, v[c] != 0u);
+                wrun += __popc(mk[c]);
+            }
+            if (lane == 0) wtot[rw] = wrun;
+            const long long ca = clock64();
+            seg_a += ca - c0;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            if constexpr (V == 0) {
+                const uint32_t cw = lane < kW ? wtot[lane] : 0u;
+                uint32_t iw = cw;
+#pragma unroll
+                for (int sh = 1; sh < 32; sh <<= 1) {
+                    const uint32_t y = __shfl_up_sync(kFull, iw, sh);
+                    if (lane >= sh) iw += y;
+                }
+                total = __shfl_sync(kFull, iw, 31);
+                wbase = __shfl_sync(kFull, iw - cw, rw);
+            } else {
+                total = 0; wbase = 0;
+#pragma unroll
+                for (int i = 0; i < kW; ++i) { const uint32_t cw = wtot[i]; wbase += i < rw ? cw : 0u; total += cw; }
+            }
+            seg_b += clock64() - c0 + (total & 1);
+            if constexpr (V != 2) {
+                uint32_t r = wbase;
+#pragma unroll
+                for (int c = 0; c < kChunks; ++c) {
+                    const uint32_t rl = r + __popc(mk[c] & lt);
+                    if (mk[c] >> lane & 1u) stage[rl] = v[c];
+                    r += __popc(mk[c]);
+                }
+            } else {
+                acc += wbase;
+            }
+        }
+        if (!(VV & 16)) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+        const long long c1 = clock64();
+        total_cyc += c1 - c0;
+        acc += total;
+        __syncthreads();
+        if (it == rounds - 1) {
+            for (int i = tid; i < kT; i += kW * 32) dump[size_t(blockIdx.x) * (kT + 1) + i] = stage[i];
+            if (tid == 0) dump[size_t(blockIdx.x) * (kT + 1) + kT] = total;
+        }
+    }
+    if (tid == 0) { cyc[blockIdx.x] = total_cyc; cyc[gridDim.x + blockIdx.x] = seg_a; cyc[2 * gridDim.x + blockIdx.x] = seg_b; }
+    if (acc == 0x12345) atomicAdd(sink, acc + stage[lane]);
+}
+
+int main() {
+    int sms;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
+    const size_t nw = size_t(64) * kT;
+    uint32_t* h = (uint32_t*)malloc(nw * 4);
+    uint64_t x = 0x9E3779B97F4A7C15ull;
+    for (size_t i = 0; i < nw; ++i) {
+        x ^= x << 13; x ^= x >> 7; x ^= x << 17;
+        h[i] = (x >> 40) & 1 ? uint32_t(x) | 1u : 0u;
+    }
+    uint32_t* d;
+    unsigned long long *cyc, *sink;
+    CK(cudaMalloc(&d, nw * 4));
+    CK(cudaMalloc(&cyc, 3 * sms * 8));
+    CK(cudaMalloc(&sink, 8));
+    CK(cudaMemcpy(d, h, nw * 4, cudaMemcpyHostToDevice));
+    const int rounds = 200;
+    uint32_t* dump;
+    CK(cudaMalloc(&dump, size_t(sms) * (kT + 1) * 4));
+    uint32_t* ref = (uint32_t*)malloc(size_t(sms) * (kT + 1) * 4);
+    uint32_t* got = (uint32_t*)malloc(size_t(sms) * (kT + 1) * 4);
+    bool have_ref = false;
+    auto run = [&](const char* name, auto kern) {
+        kern<<<sms, kW * 32>>>(d, rounds, cyc, sink, dump);
+        CK(cudaDeviceSynchronize());
+        unsigned long long hc[3 * 256];
+        CK(cudaMemcpy(hc, cyc, 3 * sms * 8, cudaMemcpyDeviceToHost));
+        double m[3] = {0, 0, 0};
+        for (int j = 0; j < 3; ++j)
+            for (int i = 0; i < sms; ++i) m[j] += double(hc[j * sms + i]) / rounds;
+        CK(cudaMemcpy(got, dump, size_t(sms) * (kT + 1) * 4, cudaMemcpyDeviceToHost));
+        if (!have_ref) { memcpy(ref, got, size_t(sms) * (kT + 1) * 4); have_ref = true; }
+        int bad = 0;
+        for (int b = 0; b < sms; ++b) {
+            const uint32_t* r = ref + size_t(b) * (kT + 1); const uint32_t* g = got + size_t(b) * (kT + 1);
+            if (r[kT] != g[kT]) { ++bad; continue; }
+            for (uint32_t i = 0; i < r[kT]; ++i) if (r[i] != g[i]) { ++bad; break; }
+        }
+        printf("%-40s %8.0f cycles per tile (warp 0: ballots done %5.0f, scan done %5.0f)  %s\n", name, m[0] / sms,
+               m[1] / sms, m[2] / sms, bad ? "MISMATCH" : "same as V0");
+    };
+    run("V0 libds ranker", rank_kernel<0>);
+    run("V1 broadcast scan", rank_kernel<1>);
+    run("V2 V1 without compaction stores", rank_kernel<2>);
+    run("V3 64-bit loads, two ballots", rank_kernel<3>);
+    run("V4 128-bit loads, four ballots", rank_kernel<4>);
+    run("V10 packed shuffle scan", rank_kernel<10>);
+    run("V10 no fence", rank_kernel<10 | 16>);
+    run("V9 chunk offsets from phase 1", rank_kernel<9>);
+    run("V9 no fence", rank_kernel<9 | 16>);
+    run("V7 chunk offsets via smem", rank_kernel<7>);
+    run("V8 chunk offsets via shuffles", rank_kernel<8>);
+    run("V7 no fence", rank_kernel<7 | 16>);
+    run("V5 loads + count, no ballots", rank_kernel<5 | 16>);
+    run("V6 loads only", rank_kernel<6 | 16>);
+    run("V1 no fence", rank_kernel<1 | 16>);
+    run("V2 no fence (ranking only)", rank_kernel<2 | 16>);
+    run("V3 no fence", rank_kernel<3 | 16>);
+    run("V4 no fence", rank_kernel<4 | 16>);
+    return 0;
+}

@@ -65,6 +65,19 @@ def main():
     for name, d in (("wait-for-lower-AGG", agg_max_lower - ev[:, 3]), ("incl-after-ready", ev[:, 4] - ready)):
         q = np.percentile(d[1:], [5, 50, 95, 99])
         print(f"{name:19s} p5 {q[0]:7.2f}  p50 {q[1]:7.2f}  p95 {q[2]:7.2f}  p99 {q[3]:7.2f}")
+    # ranker occupancy: busy = own tile (landed .. compacted), gap = until the CTA's next tile lands
+    sm = t[:, 7]
+    r1, r15 = (t[:, 1] - t0) / 1e3, (t[:, 15] - t0) / 1e3
+    busy = r15 - r1
+    gaps = []
+    for s_ in np.unique(sm):
+        idx = np.where(sm == s_)[0]
+        idx = idx[np.argsort(r1[idx])]
+        gaps.append(r1[idx[1:]] - r15[idx[:-1]])
+    gaps = np.concatenate(gaps)
+    for name, d in (("rank:busy", busy), ("rank:gap", gaps), ("rank:agg->end", r15 - ev[:, 2])):
+        q = np.percentile(d, [5, 50, 95, 99])
+        print(f"{name:13s} p5 {q[0]:7.2f}  p50 {q[1]:7.2f}  p95 {q[2]:7.2f}  p99 {q[3]:7.2f}  mean {d.mean():7.2f}")
     total = ev[:, 6] - ev[:, 0]
     print(f"{'tile':9s} p50 {np.median(total):7.2f} mean {total.mean():7.2f}")
     # how far behind the newest drawn tile is the INCL frontier, sampled over time
