@@ -37,6 +37,8 @@
 // lie in [0, (t+1)T), so no lower tile writes into a higher tile's input.
 // Deadlock freedom: look-backs wait only for lower (already drawn) tiles, and
 // a drawn tile reaches AGG without waiting on any other tile.
+#include <type_traits>
+
 #include "ds_device.cuh"
 #include "ds_internal.h"
 
@@ -645,42 +647,50 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             uint32_t wrun = 0;    // kept words of the warp's segment
 #pragma unroll
             for (int c = 0; c < kChunks; ++c) v[c] = stage[kPre + xs + 32 * c + lane];
+            // Tile-relative bounds: only tile 0 (the array's first word, the lead
+            // words below p.lo) and the last tile need the guarded pass; every
+            // other tile takes the branch-free pass (same ops, no range checks).
+            const uint32_t xlo = tb < p.lo ? uint32_t(p.lo - tb) : 0u;
+            const uint32_t xhi = tb + kT <= p.hi ? uint32_t(kT) : uint32_t(p.hi - tb);
+            const bool guarded = !full || t == 0;
+            auto count_pass = [&](auto guard_tag) {
+                constexpr bool G = decltype(guard_tag)::value;
 #pragma unroll
-            for (int c = 0; c < kChunks; ++c) {
-                const int x = xs + 32 * c + lane;
-                bool kp;
-                if constexpr (Op::kWide) {
-                    // element = (even word, odd word) = lanes (2m, 2m+1) of the chunk
-                    const uint32_t partner = __shfl_xor_sync(kFull, v[c], 1);
-                    const uint32_t lo = (lane & 1) ? partner : v[c], hi = (lane & 1) ? v[c] : partner;
-                    const int xe = x - (lane & 1);  // the element's first word
-                    if constexpr (Op::kUnique) {
-                        kp = lo != stage[kPre + xe - 2] || hi != stage[kPre + xe - 1];
-                        if (tb + xe == p.lo) kp = true;  // the array's first element
+                for (int c = 0; c < kChunks; ++c) {
+                    const uint32_t x = uint32_t(xs + 32 * c + lane);
+                    bool kp;
+                    if constexpr (Op::kWide) {
+                        // element = (even word, odd word) = lanes (2m, 2m+1) of the chunk
+                        const uint32_t partner = __shfl_xor_sync(kFull, v[c], 1);
+                        const uint32_t lo = (lane & 1) ? partner : v[c], hi = (lane & 1) ? v[c] : partner;
+                        const uint32_t xe = x - (lane & 1);  // the element's first word
+                        if constexpr (Op::kUnique) {
+                            kp = lo != stage[kPre + xe - 2] || hi != stage[kPre + xe - 1];
+                            if (G && t == 0 && xe == xlo) kp = true;  // the array's first element
+                        } else {
+                            kp = Op::keep2((uint64_t(hi) << 32) | lo, (uint64_t(p.value_hi) << 32) | p.value);
+                        }
+                    } else if constexpr (Op::kUnique) {
+                        // previous word straight from the staged tile; x == 0 reads
+                        // the word before the tile
+                        kp = v[c] != stage[kPre + x - 1];
+                        if (G && t == 0 && x == xlo) kp = !has_hprev || v[c] != hprev;  // the array's first word (R18)
                     } else {
-                        kp = Op::keep2((uint64_t(hi) << 32) | lo, (uint64_t(p.value_hi) << 32) | p.value);
+                        kp = Op::keep(v[c], p.value);
                     }
-                } else if constexpr (Op::kUnique) {
-                    // previous word straight from the staged tile; x == 0 reads
-                    // the word before the tile
-                    kp = v[c] != stage[kPre + x - 1];
-                    if (tb + x == p.lo) kp = !has_hprev || v[c] != hprev;  // the array's first word (R18)
-                } else {
-                    kp = Op::keep(v[c], p.value);
+                    if (G) kp = kp && x >= xlo && x < xhi;
+                    const uint32_t mk = __ballot_sync(kFull, kp);
+                    if constexpr (kMaskRegs) {
+                        mkr[c] = mk;
+                        if constexpr (kRc) rc[c] = wrun;  // kept words of the segment before chunk c
+                    } else if (lane == c) {
+                        mymask = mk;
+                    }
+                    wrun += __popc(mk);
                 }
-                if (!full) {
-                    const uint64_t e = tb + x;
-                    kp = kp && e >= p.lo && e < p.hi;
-                }
-                const uint32_t mk = __ballot_sync(kFull, kp);
-                if constexpr (kMaskRegs) {
-                    mkr[c] = mk;
-                    if constexpr (kRc) rc[c] = wrun;  // kept words of the segment before chunk c
-                } else if (lane == c) {
-                    mymask = mk;
-                }
-                wrun += __popc(mk);
-            }
+            };
+            if (guarded) count_pass(std::true_type{});
+            else count_pass(std::false_type{});
             if (lane == 0) meta[o].wtot[rw] = wrun;
             if (rt == 0) trace_event(p.trace, t, 13, globaltimer());
             named_bar_sync(gbar, kRT);  // warp totals written; every ranker holds its words
