@@ -640,7 +640,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             // ballot of chunk c is kept by lane c (one register instead of kChunks).
             const int xs = kSeg * rw;
             constexpr bool kMaskRegs = kChunks <= 16;  // else chunk c's mask is held by lane c
-            constexpr bool kRc = kMaskRegs && !PART && !Op::kUnique;  // chunk offsets from the count (registers)
+            constexpr bool kRc = kMaskRegs && !PART;  // chunk offsets from the count (registers)
             uint32_t v[kChunks];
             uint32_t mkr[kMaskRegs ? kChunks : 1], rc[kRc ? kChunks : 1];
             uint32_t mymask = 0;  // lane c: keep mask of chunk c (!kMaskRegs)
