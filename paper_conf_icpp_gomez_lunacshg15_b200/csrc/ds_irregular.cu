@@ -19,7 +19,7 @@
 //                       below the lane + a scan of the 16 warp totals); the
 //                       kept words are compacted in place, 32 consecutive
 //                       words per store
-//   6 resolver warps a5 (one per stage) decoupled look-back over 128
+//   6 resolver warps a5 (one per stage) decoupled look-back over 32
 //                       predecessors per round trip, started as soon as the
 //                       ticket is drawn (it needs no data), then INCL; the last
 //                       tile writes out_n (a8).  This replaces the serial flag
@@ -210,13 +210,14 @@ __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) 
     return false;
 }
 
-// a5: decoupled look-back by one warp over 512 predecessors per round trip.
+// a5: decoupled look-back by one warp over 32 * kLB predecessors per round trip
+// (kLB = 1: fewer status sectors per poll beat a wider window).
 // Slot (m, lane) examines tile base - (32m + lane): every load instruction
 // reads 32 consecutive status words.  Waits only for the tiles up to the
 // nearest INCL predecessor.  Ends with one acquire fence per lane and a
 // __syncwarp so lane 0's later release is cumulative over all lanes.
 #ifndef DS_IRR_LB
-#define DS_IRR_LB 4
+#define DS_IRR_LB 1
 #endif
 constexpr int kLB = DS_IRR_LB;  // look-back slots per lane (32 * kLB tiles per round)
 #ifndef DS_IRR_REFRESH
