@@ -523,10 +523,16 @@ __device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph
 // mbarrier wait that also returns (false) once the CTA's work is known to
 // end before ring position k (the resolvers take alternate positions, so the
 // one not holding the end marker is released this way).
+// Suspend-time hint of those waits: it bounds how long a warp parked on a
+// position past the end keeps the CTA (and so the launch) alive.
+#ifndef DS_IRR_END_POLL_NS
+#define DS_IRR_END_POLL_NS 1000
+#endif
+constexpr uint32_t kEndPollNs = DS_IRR_END_POLL_NS;
 __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
                                                  const volatile uint32_t* s_end, uint32_t k) {
     while (true) {
-        if (mbar_try_wait(bar, parity, 20000u)) return true;
+        if (mbar_try_wait(bar, parity, kEndPollNs)) return true;
         // Strictly beyond the end marker: the position holding the marker
         // itself still gets its arrival and must pass it on.
         if (*s_end < k) return false;

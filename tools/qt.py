@@ -52,6 +52,14 @@ def run(spec):
         a = dsgen.compact_input(n, f, dsgen.seed_for(0), device=dev)
         timeit(f"compact 1M f={f}", a, lambda w, d: libds.ds_compact_ex(w, n, 0, d, None), lambda m: 4 * (n + m),
                reps=30)
+    elif op == "c1b2b":  # 20 back-to-back calls between the events (launch-to-launch time)
+        n = 1 << 20
+        a = dsgen.compact_input(n, f, dsgen.seed_for(0), device=dev)
+
+        def calls(w, d):
+            for _ in range(20):
+                libds.ds_compact_ex(w, n, 0, d, None)
+        timeit(f"compact 1M f={f} x20", a, calls, lambda m: 20 * 4 * (n + m), reps=10)
     elif op == "select":
         n = 1 << 28
         a = dsgen.select_input(n, 3, device=dev)
