@@ -153,13 +153,19 @@ __device__ __forceinline__ void wait_loaded(const uint64_t* __restrict__ status,
     __syncwarp();
 }
 
-constexpr int kConsumerWarps = 8;
+#ifndef DS_REG_CONSUMER_WARPS
+#define DS_REG_CONSUMER_WARPS 16
+#endif
+#ifndef DS_REG_STAGES
+#define DS_REG_STAGES 3
+#endif
+constexpr int kConsumerWarps = DS_REG_CONSUMER_WARPS;
 constexpr int kCT = 32 * kConsumerWarps;  // consumer threads
-constexpr int kItems = 32;                // output words per consumer thread
+constexpr int kItems = 8192 / kCT;        // output words per consumer thread
 constexpr int kVec = kItems / 4;
 constexpr int kT = kCT * kItems;          // 8192 output words = 32 KB per tile
 constexpr int kStageWords = kT + 512;     // staged source span cap (words)
-constexpr int kStages = 3;
+constexpr int kStages = DS_REG_STAGES;
 constexpr int kThreads = 32 * (2 + kConsumerWarps);  // producer, publisher, consumers
 constexpr size_t kSmem = size_t(kStages) * kStageWords * 4;
 

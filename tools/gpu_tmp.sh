@@ -1,3 +1,2 @@
-timeout 300 python tools/qt.py c1 c1b2b 2>&1 | grep -v Warn
-timeout 300 nsys --version 2>/dev/null
-timeout 300 ncu --metrics gpu__time_duration.sum,sm__cycles_active.avg,smsp__cycles_active.avg --csv -k regex:irregular -c 3 python tools/qt.py c1 2>/dev/null | tail -6
+L=$PWD/paper_conf_icpp_gomez_lunacshg15_b200/lib
+for v in libds libds_rc16 libds_rc16s2 libds_rs2; do LIBDS_PATH=$L/$v.so timeout 300 python tools/qt.py pad unpad pad12k; done 2>&1 | grep -v Warn

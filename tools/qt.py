@@ -80,6 +80,11 @@ def run(spec):
             libds.ds_pad(a, R, C, NC, 4)
             timeit("unpad 4000x4000->3990", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, 4, None),
                    lambda m: 4 * (2 * R * C), reps=30)
+    elif op == "pad12k":
+        R, C, NC = 12000, 11999, 12000
+        a = dsgen.matrix_input(R, C, NC, 4, device=dev)
+        timeit("pad 12000x11999->12000", a, lambda w, d: libds.ds_pad_ex(w, R, C, NC, 4, None, None),
+               lambda m: 4 * (R * C + R * NC))
     else:
         raise SystemExit(f"unknown op {op}")
     torch.cuda.empty_cache()
