@@ -23,9 +23,12 @@ namespace ds {
 namespace {
 
 constexpr int64_t kNoTileB = -1;
-constexpr int kBConsumerWarps = 8;
+#ifndef DS_REGB_CONSUMER_WARPS
+#define DS_REGB_CONSUMER_WARPS 16
+#endif
+constexpr int kBConsumerWarps = DS_REGB_CONSUMER_WARPS;
 constexpr int kBCT = 32 * kBConsumerWarps;
-constexpr int kBChunks = 8;                   // 16-byte chunks per consumer thread
+constexpr int kBChunks = 2048 / kBCT;         // 16-byte chunks per consumer thread
 constexpr int kTB = kBCT * kBChunks * 16;     // 32768 output bytes per tile
 constexpr int kBStageBytes = kTB + 2048;      // staged source span cap
 constexpr int kBStageAlloc = kBStageBytes + 32;  // vector reads may pass the span by 16 bytes

@@ -80,6 +80,16 @@ def run(spec):
             libds.ds_pad(a, R, C, NC, 4)
             timeit("unpad 4000x4000->3990", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, 4, None),
                    lambda m: 4 * (2 * R * C), reps=30)
+    elif op in ("padb1", "padb2", "unpadb1", "unpadb2"):  # sub-word elements, byte-granular kernel
+        R, C, NC = 4000, 3990, 4000
+        eb = int(op[-1])
+        a = torch.randint(0, 256, (R * NC * eb,), dtype=torch.uint8, device=dev)
+        if op.startswith("pad"):
+            timeit(f"pad {R}x{C}->{NC} eb={eb}", a, lambda w, d: libds.ds_pad_ex(w, R, C, NC, eb, None, None),
+                   lambda m: eb * (R * C + R * NC), reps=30)
+        else:
+            timeit(f"unpad {R}x{NC}->{C} eb={eb}", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, eb, None),
+                   lambda m: eb * (2 * R * C), reps=30)
     elif op == "pad12k":
         R, C, NC = 12000, 11999, 12000
         a = dsgen.matrix_input(R, C, NC, 4, device=dev)
