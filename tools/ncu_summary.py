@@ -66,6 +66,54 @@ def num(m, key):
     return x * mult
 
 
+def role_samples(rep, src_file):
+    """Warp-state samples per role of the irregular kernel, from the cuda,sass
+    source view (-lineinfo + --import-source): lines of ds_irregular.cu are
+    attributed to the function / role section that contains them, by the
+    section markers in the source; inlined helpers from other files count as
+    'helpers'.  'look-back' = the decoupled look-back's poll loop (the
+    flag-spin of SURVEY 8(d))."""
+    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+                         capture_output=True, text=True).stdout
+    with open(src_file) as fh:
+        lines = fh.read().split("\n")
+
+    def find(pat):
+        return next((i + 1 for i, x in enumerate(lines) if pat in x), None)
+    marks = sorted((v, k) for k, v in {
+        "look-back": find("uint64_t lookback("), "look-back (local chain)": find("uint64_t lookback_window("),
+        "store helpers": find("void store_segment("), "kernel setup": find("mbar_wait_or_end("),
+        "producer": find("---- producer"), "rankers": find("---- ranker warps"),
+        "resolvers": find("---- resolver warps"), "storers": find("---- storer warps"),
+        "host": find("struct LaunchCache")}.items() if v)
+    roles, cur_file, col = {}, None, None
+    for r in csv.reader(io.StringIO(out)):
+        if not r:
+            continue
+        if r[0] in ("File Path", "File Name"):
+            cur_file = r[1]
+            continue
+        if r[0] == "Line No":
+            col = r.index("Warp Stall Sampling (All Samples)")
+            continue
+        if col is None or not r[0].isdigit():
+            continue
+        try:
+            smp = int(r[col])
+        except ValueError:
+            continue
+        if cur_file and os.path.basename(cur_file) == os.path.basename(src_file):
+            ln = int(r[0])
+            role = "other"
+            for start, name in marks:
+                if ln >= start:
+                    role = name
+        else:
+            role = "helpers (" + os.path.basename(cur_file or "?") + ")"
+        roles[role] = roles.get(role, 0) + smp
+    return roles
+
+
 def main():
     rnd = sys.argv[1]
     src = sys.argv[2] if len(sys.argv) > 2 else os.path.join(ROOT, "gpurun_out")
@@ -111,6 +159,30 @@ def main():
                f"(ncu's own peak), warps active {head['sm__warps_active.avg.pct_of_peak_sustained_active']} %, "
                f"registers {head['launch__registers_per_thread']}, grid {head['launch__grid_size']} x "
                f"{head['launch__block_size']}", ""]
+        if os.path.exists(rep):
+            roles = role_samples(rep, os.path.join(ROOT, "paper_conf_icpp_gomez_lunacshg15_b200", "csrc",
+                                                   "ds_irregular.cu"))
+            tot = sum(roles.values())
+            if tot:
+                summary["warp_samples_by_role"] = roles
+                summary["flag_spin_fraction"] = roles.get("look-back", 0) / tot
+                md += ["## Warp-state samples by role (source view, all warps of the headline kernel)", "",
+                       "| role | samples | share |", "|---|---|---|"]
+                for k, v in sorted(roles.items(), key=lambda kv: -kv[1]):
+                    md.append(f"| {k} | {v} | {v / tot:.1%} |")
+                md += ["", f"Flag-spin fraction (samples in the look-back poll loop / all samples): "
+                       f"{summary['flag_spin_fraction']:.1%}.  The look-back runs on dedicated resolver "
+                       "warps, so these samples are parked pollers, not stalled data movers; the "
+                       "rankers' share is the busy fraction of the ranking step.", ""]
+        ld_sec = num(m, "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum")
+        ld_req = num(m, "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum")
+        st_sec = num(m, "l1tex__t_sectors_pipe_lsu_mem_global_op_st.sum")
+        st_req = num(m, "l1tex__t_requests_pipe_lsu_mem_global_op_st.sum")
+        if ld_req and st_req:
+            summary["lsu_sectors_per_request"] = {"ld": ld_sec / ld_req, "st": st_sec / st_req}
+            md += [f"LSU sectors/request: loads {ld_sec / ld_req:.1f} (the status polls: 32 statuses 64 B apart "
+                   f"per warp load), stores {st_sec / st_req:.1f} (status words and the <= 6 scalar head/tail "
+                   "words per tile).  The tile data moves through TMA bulk copies, not the LSU.", ""]
     with open(os.path.join(prof, "ncu_summary.json"), "w") as fh:
         json.dump(summary, fh, indent=1)
     with open(os.path.join(prof, f"ncu_{rnd}.md"), "w") as fh:
