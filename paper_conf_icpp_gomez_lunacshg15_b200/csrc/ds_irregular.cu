@@ -219,7 +219,12 @@ __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) 
 #ifndef DS_IRR_LB
 #define DS_IRR_LB 1
 #endif
-constexpr int kLB = DS_IRR_LB;  // look-back slots per lane (32 * kLB tiles per round)
+constexpr int kLB = DS_IRR_LB;  // look-back slots per lane (kLBW * kLB tiles per round)
+#ifndef DS_IRR_LBW
+#define DS_IRR_LBW 32
+#endif
+constexpr int kLBW = DS_IRR_LBW;  // lanes that read statuses (window width per slot row)
+static_assert(kLBW >= 1 && kLBW <= 32, "look-back lanes");
 #ifndef DS_IRR_REFRESH
 #define DS_IRR_REFRESH 1
 #endif
@@ -247,6 +252,7 @@ constexpr bool DBG_NO_PFENCE = DS_DEBUG_BISECT & 1, DBG_NO_PUBLISH = DS_DEBUG_BI
 #define DS_IRR_HELP 0
 #endif
 constexpr bool kHelp = DS_IRR_HELP;  // publish INCL for the nearest 32 AGG predecessors
+static_assert(!kHelp || kLBW == 32, "helper INCLs assume the 32-lane window");
 
 __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint32_t tile,
                                              uint32_t epoch, int lane, uint64_t* trace) {
@@ -258,14 +264,15 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
     while (true) {
         uint64_t s[kLB];
         uint32_t okm = 0;  // bit m: slot m holds a current status
+        const bool act = lane < kLBW;  // lanes of the window (the rest read as empty, current)
 #pragma unroll
         for (int m = 0; m < kLB; ++m) {
-            const int64_t idx = base - (32 * m + lane);
-            s[m] = idx >= 0 ? ld_relaxed_gpu(status_ptr(status, idx)) : make_status(kStateIncl, epoch, 0);
+            const int64_t idx = base - (kLBW * m + lane);
+            s[m] = !act ? 0ull : idx >= 0 ? ld_relaxed_gpu(status_ptr(status, idx)) : make_status(kStateIncl, epoch, 0);
         }
 #pragma unroll
         for (int m = 0; m < kLB; ++m)
-            if (status_current(s[m], epoch)) okm |= 1u << m;
+            if (!act || status_current(s[m], epoch)) okm |= 1u << m;
         if (rounds++ == 0 && lane == 0) trace_event(trace, tile, 10, globaltimer());
         uint32_t ns = kPollMinNs;
         uint32_t M, L;  // nearest INCL at slot M, lane L (M == kLB: none this round)
@@ -290,9 +297,9 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
 #pragma unroll
             for (int m = 0; m < kLB; ++m) {
                 const bool pending = !(okm >> m & 1u);
-                const bool refresh = m < kRefreshRows && !pending && status_state(s[m]) != kStateIncl;
+                const bool refresh = act && m < kRefreshRows && !pending && status_state(s[m]) != kStateIncl;
                 if ((need >> m & 1u) && (pending || refresh)) {
-                    const int64_t idx = base - (32 * m + lane);
+                    const int64_t idx = base - (kLBW * m + lane);
                     if (idx >= 0) {
                         s[m] = ld_relaxed_gpu(status_ptr(status, idx));
                         okm = status_current(s[m], epoch) ? (okm | 1u << m) : (okm & ~(1u << m));
@@ -316,7 +323,7 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
             excl += __shfl_sync(kFull, inc, L);
             break;
         }
-        base -= 32 * kLB;
+        base -= kLBW * kLB;
     }
     if (kHelp) {
         // The walk fixed the inclusive prefix of every tile it summed: for the
