@@ -204,6 +204,30 @@ def bench_rows(peak, flush):
         irregular("compact", f"C4 1G f32 f={f}", src,
                   lambda w: libds.ds_compact_ex(w, n, 0, d_n, None), reps=3)
         del src
+    # 8(f)-3: 8-byte elements (int64 compaction, 256M elements = 2 GiB, 50 % kept)
+    n = 1 << 28
+    h = dsgen.hash_range(dsgen.seed_for(6), 0, n, device="cuda")
+    src = torch.where(dsgen._hi32(h) < dsgen.keep_threshold(0.5), h | 1, torch.zeros_like(h))
+    del h
+    work = torch.empty_like(src)
+    ms = timed(lambda: libds.ds_compact64_ex(work, n, 0, d_n, None), s, restore=lambda: work.copy_(src),
+               flush=flush, reps=3)
+    m = int(d_n.item())
+    row("compact64", "256M int64 f=0.5 (8-byte elements)", ms, 8 * (n + m), {"n": n, "out_n": m})
+    del src, work
+    # 8(f)-4: sub-word elements, C2 shape (byte-granular kernel for 1-byte rows of
+    # 3990 bytes; 2-byte rows are whole words and take the word kernel)
+    R, C, NC = 4000, 3990, 4000
+    for eb in (1, 2):
+        src = torch.randint(0, 256, (R * NC * eb,), dtype=torch.uint8, device="cuda")
+        work = torch.empty_like(src)
+        ms = timed(lambda: libds.ds_pad_ex(work, R, C, NC, eb, None, None), s,
+                   restore=lambda: work.copy_(src), flush=flush, reps=20)
+        row("pad", f"C2 shape {R}x{C}->{NC} eb={eb}", ms, eb * (R * C + R * NC))
+        ms = timed(lambda: libds.ds_unpad_ex(work, R, NC, C, eb, None), s,
+                   restore=lambda: work.copy_(src), flush=flush, reps=20)
+        row("unpad", f"C2 shape {R}x{NC}->{C} eb={eb}", ms, eb * 2 * R * C)
+        del src, work
     return rows
 
 
