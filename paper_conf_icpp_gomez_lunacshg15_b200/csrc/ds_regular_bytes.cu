@@ -50,6 +50,7 @@ struct RegBParams {
     uint32_t draws;
     uint64_t* status;
     uint64_t* ctrl;
+    uint64_t* trace;       // diagnostics: per-tile events, or null (as the word kernel)
 };
 
 struct TileGeomB {
@@ -136,6 +137,28 @@ __device__ __forceinline__ void wait_loaded_b(const uint64_t* __restrict__ statu
     __syncwarp();
 }
 
+// 16 consecutive bytes of the stage starting at byte offset sidx (any phase):
+// two aligned 16-byte shared loads, a word select and four funnel shifts.
+// Reads up to 31 bytes past sidx (inside the stage allocation's slack).
+__device__ __forceinline__ void load16(const uint32_t* stage32, int32_t sidx, uint32_t out[4]) {
+    const int32_t w = sidx >> 2;
+    const uint32_t bph = uint32_t(sidx) & 3u, wph = uint32_t(w) & 3u;
+    const u32x4 A = *reinterpret_cast<const u32x4*>(stage32 + (w & ~3));
+    const u32x4 B = *reinterpret_cast<const u32x4*>(stage32 + (w & ~3) + 4);
+    const uint32_t a[8] = {A.x, A.y, A.z, A.w, B.x, B.y, B.z, B.w};
+    uint32_t h[5];
+#pragma unroll
+    for (int j = 0; j < 5; ++j) {
+        uint32_t v = a[j];
+#pragma unroll
+        for (uint32_t q = 1; q < 4; ++q)
+            if (wph == q) v = a[j + q];
+        h[j] = v;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) out[j] = __funnelshift_r(h[j], h[j + 1], 8 * bph);
+}
+
 __device__ __forceinline__ uint8_t ldg_u8(const uint8_t* p) {
     uint16_t v;
     asm volatile("ld.global.L1::no_allocate.u8 %0, [%1];" : "=h"(v) : "l"(p));
@@ -201,6 +224,8 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
             const int64_t kt = PAD ? int64_t(p.ntiles) - 1 - t : int64_t(t);
             if (lane == 0) {
                 debug_delay(uint64_t(kt), 0);
+                trace_event(p.trace, uint64_t(kt), 0, globaltimer());
+                trace_event(p.trace, uint64_t(kt), 7, smid());
                 tile_geometry_b<PAD>(p, kt, geo[s]);
                 geo_epoch[s] = epoch;
                 if (geo[s].bytes) {
@@ -224,8 +249,10 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
             const int64_t kt = geo[s].k;
             if (lane == 0) {
                 if (kt != kNoTileB) {
+                    trace_event(p.trace, uint64_t(kt), 1, globaltimer());
                     debug_delay(uint64_t(kt), 1);
                     publish_status(status_ptr(p.status, kt), make_status(kStateLoaded, geo_epoch[s], 0));
+                    trace_event(p.trace, uint64_t(kt), 2, globaltimer());
                 }
                 mbar_arrive(&bar_loaded[s]);
             }
@@ -242,7 +269,11 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
             mbar_wait(&bar_loaded[s], (k / kBStages) & 1);
             const TileGeomB g = geo[s];
             if (g.k == kNoTileB) break;
-            if (warp == 2 && g.win_lo <= g.win_hi) wait_loaded_b(p.status, g.win_lo, g.win_hi, geo_epoch[s], lane);
+            if (warp == 2) {
+                if (lane == 0) trace_event(p.trace, uint64_t(g.k), 3, globaltimer());
+                if (g.win_lo <= g.win_hi) wait_loaded_b(p.status, g.win_lo, g.win_hi, geo_epoch[s], lane);
+                if (lane == 0) trace_event(p.trace, uint64_t(g.k), 4, globaltimer());
+            }
             const int64_t V0 = g.k * kTB;
             const int32_t soff = int32_t(g.slo + mis - g.sb);
             uint32_t o[kBChunks][4];
@@ -254,25 +285,42 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
                 uint32_t dr = fastdiv(t, p.div_nc);
                 uint32_t col = t - dr * p.NCb;
                 const bool whole = vq >= g.q0 && vq + 16 <= g.q1;
-                if (whole && g.bytes && col + 16 <= data_cols) {
+                // fast path: the chunk lies in one output row and starts in its data;
+                // for pad it may end in the row's fill (merged below)
+                if (whole && g.bytes && col < data_cols && col + 16 <= (PAD ? p.NCb : data_cols)) {
                     // 16 consecutive source bytes at byte offset sidx of the stage
                     const int32_t sidx = g.base_rel + int32_t(dr * p.Cb + col) + soff;
-                    const int32_t w = sidx >> 2;
-                    const uint32_t bph = uint32_t(sidx) & 3u, wph = uint32_t(w) & 3u;
-                    const u32x4 A = *reinterpret_cast<const u32x4*>(stage32 + (w & ~3));
-                    const u32x4 B = *reinterpret_cast<const u32x4*>(stage32 + (w & ~3) + 4);
-                    const uint32_t a[8] = {A.x, A.y, A.z, A.w, B.x, B.y, B.z, B.w};
-                    uint32_t h[5];
+                    load16(stage32, sidx, o[i]);
+                    if (PAD && col + 16 > data_cols) {
+                        // the row's last nd data bytes, then its fill: the bytes read past
+                        // the data end (inside the staged span + slack) are replaced
+                        const int32_t nd = int32_t(data_cols - col);
+                        const uint32_t f0 = p.fill[0], f1 = p.fill[p.eb - 1];
+                        uint32_t pat = (col & 1u) && p.eb == 2 ? (f1 | f0 << 8) : (f0 | f1 << 8);
+                        pat |= pat << 16;
 #pragma unroll
-                    for (int j = 0; j < 5; ++j) {
-                        uint32_t v = a[j];
-#pragma unroll
-                        for (uint32_t q = 1; q < 4; ++q)
-                            if (wph == q) v = a[j + q];
-                        h[j] = v;
+                        for (int j = 0; j < 4; ++j) {
+                            const int32_t keep = nd - 4 * j;
+                            const uint32_t m = keep >= 4 ? 0xffffffffu : keep <= 0 ? 0u : (1u << (8 * keep)) - 1u;
+                            o[i][j] = (o[i][j] & m) | (pat & ~m);
+                        }
                     }
+                    continue;
+                }
+                if (!PAD && whole && g.bytes && p.NCb >= 16 && col + 16 > p.NCb) {
+                    // unpad: the end of output row r, then the start of row r + 1, whose
+                    // source follows the Cb - NCb dropped bytes: two 16-byte reads, merged
+                    const int32_t sidx = g.base_rel + int32_t(dr * p.Cb + col) + soff;
+                    uint32_t o1[4], o2[4];
+                    load16(stage32, sidx, o1);
+                    load16(stage32, sidx + int32_t(p.Cb - p.NCb), o2);
+                    const int32_t nd = int32_t(p.NCb - col);  // bytes of row r (1..15)
 #pragma unroll
-                    for (int j = 0; j < 4; ++j) o[i][j] = __funnelshift_r(h[j], h[j + 1], 8 * bph);
+                    for (int j = 0; j < 4; ++j) {
+                        const int32_t keep = nd - 4 * j;
+                        const uint32_t m = keep >= 4 ? 0xffffffffu : keep <= 0 ? 0u : (1u << (8 * keep)) - 1u;
+                        o[i][j] = (o1[j] & m) | (o2[j] & ~m);
+                    }
                     continue;
                 }
                 if (PAD && whole && col >= p.Cb && col + 16 <= p.NCb) {  // 16 fill bytes
@@ -293,7 +341,7 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
                             col = g.col0;
                         }
                         if (!g.bytes && g.span > 0) val = stage[uint32_t(q - g.q0)];
-                        else if (PAD && col >= p.Cb) val = p.fill[col % p.eb];
+                        else if (PAD && col >= p.Cb) val = p.fill[p.eb == 2 ? (col & 1u) : 0u];
                         else val = stage[g.base_rel + int32_t(dr * p.Cb + col) + soff];
                     }
                     wv[j >> 2] |= val << (8 * (j & 3));
@@ -309,6 +357,7 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
             if (lane == 0) mbar_arrive(&bar_empty[s]);
             if (ct == 0) debug_delay(uint64_t(g.k), 2);
             named_bar_sync(1, kBCT);  // the window wait precedes every store
+            if (ct == 0) trace_event(p.trace, uint64_t(g.k), 5, globaltimer());
 #pragma unroll
             for (int i = 0; i < kBChunks; ++i) {
                 const int64_t u = V0 + 16 * int64_t(i * kBCT + ct);  // virtual byte
@@ -321,6 +370,7 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
                             stg_u8(p.abase + u + j, uint8_t(o[i][j >> 2] >> (8 * (j & 3))));
                 }
             }
+            if (ct == 0) trace_event(p.trace, uint64_t(g.k), 6, globaltimer());
         }
     }
 }
@@ -378,6 +428,7 @@ cudaError_t launch_regular_bytes(const RegBytesArgs& a, Workspace& ws, cudaStrea
     p.fill[0] = a.fill[0];
     p.fill[1] = a.fill[1];
     p.ntiles = uint32_t(regular_bytes_tiles(a));
+    p.trace = debug_trace(p.ntiles);
     p.status = ws.status;
     p.ctrl = ws.ctrl;
     count_launch();

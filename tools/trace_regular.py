@@ -18,15 +18,22 @@ T = 8192
 def main():
     op = sys.argv[1]
     R, C, NC = (int(x) for x in sys.argv[2:5])
-    src = dsgen.matrix_input(R, C, NC, 4, device="cuda")
+    eb = int(sys.argv[5]) if len(sys.argv) > 5 else 4
+    global T
+    if eb in (1, 2) and (C * eb) % 4:  # byte-granular kernel: 32 KB output tiles
+        T = 32768 // eb
+    if eb == 4:
+        src = dsgen.matrix_input(R, C, NC, 4, device="cuda")
+    else:
+        src = torch.randint(0, 256, (R * max(C, NC) * eb,), dtype=torch.uint8, device="cuda")
     if op == "unpad":
         libds.ds_pad(src, R, NC, C, 4) if False else None
     work = torch.empty_like(src)
     out_words = R * NC
     ntiles = (out_words + T - 1) // T
     tr = torch.zeros(ntiles * 16, dtype=torch.int64, device="cuda")
-    fn = (lambda: libds.ds_pad_ex(work, R, C, NC, 4, None, None)) if op == "pad" else \
-         (lambda: libds.ds_unpad_ex(work, R, C, NC, 4, None))
+    fn = (lambda: libds.ds_pad_ex(work, R, C, NC, eb, None, None)) if op == "pad" else \
+         (lambda: libds.ds_unpad_ex(work, R, C, NC, eb, None))
     for rep in range(3):
         work.copy_(src)
         torch.cuda.synchronize()
@@ -38,7 +45,7 @@ def main():
     t0 = t[:, 0].min()
     ev = (t[:, :7] - t0) / 1e3
     span = ev[:, 6].max()
-    nbytes = 4 * (R * C + R * NC) if op == "pad" else 8 * R * NC
+    nbytes = eb * (R * C + R * NC) if op == "pad" else 2 * eb * R * NC
     print(f"{op} {R}x{C}->{NC} tiles={ntiles} span={span:.1f} us  {nbytes / span / 1e3:.0f} GB/s")
     for k, name in enumerate(["load", "publish", "->consumers", "window", "gather", "store"]):
         d = ev[:, k + 1] - ev[:, k]
