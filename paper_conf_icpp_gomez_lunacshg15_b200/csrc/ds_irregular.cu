@@ -181,6 +181,8 @@ constexpr int kAlignW = DS_IRR_ALIGN;    // stage alignment in words (32 = 128 b
 constexpr int kStageWords = (kT + kPre + 4 + kAlignW - 1) / kAlignW * kAlignW;
 constexpr size_t kSmem = size_t(kInStages) * kStageWords * 4 + 128;  // + runtime alignment slack
 static_assert(kPre % 4 == 0 && kPre >= 4, "boundary words keep 16-byte alignment");
+static_assert(!DS_IRR_BULK_STORE || kStageWords >= kT + kPre + 8,
+              "re-phase writes whole chunks up to 6 words past a segment");
 static_assert(kThreads <= 1024, "CTA size");
 static_assert(kSlots >= kInStages, "a slot per input stage at least");
 static_assert(kSlots % kResolvers == 0, "a slot is always served by the same resolver");
@@ -838,30 +840,55 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             // kept word would be written onto itself, so the stores are skipped.
             const bool identity = !PART && p.tbase == p.abase && meta[o].excl == vs0 - p.lo && A == ve0 - vs0;
 #ifndef DS_DEBUG_NO_STORE  // timing experiment only: no output written
-            if (PART || !kBulkStore) {
+            // Bulk-store cnt words that sit at seg[off + r] (off % 4 == 0 or the
+            // words before them are dead) to base[d0 + r]: re-phase them in shared
+            // memory to d0's 16-byte phase, one TMA bulk store of the aligned
+            // interior, scalar head and tail (<= 3 words each).
+            auto bulk_segment = [&](uint32_t* base, uint64_t d0, uint32_t cnt, uint32_t off) {
+                const uint64_t d1 = d0 + cnt;
+                const uint32_t sh = (uint32_t(d0) - off) & 3u;  // shift that gives word r phase d0 + r
+                uint32_t* const b = seg + (off & ~3u);          // aligned start of the moved block
+                if (sh) rephase<kST>(b, cnt + (off & 3u), sh, st);  // word off + r -> off + sh + r
+                const uint32_t* const w = seg + off + sh;        // word r now at w[r], phase of d0 + r
+                const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
+                if (g1 > g0) {
+                    fence_proxy_async_smem();  // re-phased words -> visible to the bulk engine
+                    named_bar_sync(2, kST);
+                    if (st == 0) bulk_s2g(base + g0, w + uint32_t(g0 - d0), uint32_t(g1 - g0) * 4u);
+                    if (st < 3 && d0 + st < g0) stg_stream(base + d0 + st, w[st]);
+                    if (st >= 3 && st < 6 && g1 + (st - 3) < d1)
+                        stg_stream(base + g1 + (st - 3), w[uint32_t(g1 - d0) + (st - 3)]);
+                } else {
+                    named_bar_sync(2, kST);
+                    if (uint32_t(st) < cnt) stg_stream(base + d0 + st, w[st]);  // cnt < 8
+                }
+            };
+            if (!kBulkStore) {
                 if (!identity) store_segment<kST>(p.tbase, p.tlo + meta[o].excl, A, seg, 0, st);
                 if (PART) {
                     const uint64_t excl_f = (vs0 - p.lo) - meta[o].excl;
                     store_segment<kST>(p.fbase, p.flo + excl_f, uint32_t(ve0 - vs0) - A, seg, int32_t(A), st);
                 }
-            } else if (!identity && A > 0) {
-                const uint64_t d0 = p.tlo + meta[o].excl, d1 = d0 + A;
-                const uint32_t ph = uint32_t(d0) & 3u;
-                if (ph) rephase<kST>(seg, A, ph, st);  // word r -> seg[ph + r]
-                const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
-                if (g1 > g0) {
-                    fence_proxy_async_smem();  // re-phased words -> visible to the bulk engine
-                    named_bar_sync(2, kST);
-                    if (st == 0)
-                        bulk_s2g(p.tbase + g0, seg + ph + uint32_t(g0 - d0), uint32_t(g1 - g0) * 4u);
-                    // head [d0, g0) and tail [g1, d1): at most 3 words each
-                    if (st < 3 && d0 + st < g0) stg_stream(p.tbase + d0 + st, seg[ph + st]);
-                    if (st >= 3 && st < 6 && g1 + (st - 3) < d1)
-                        stg_stream(p.tbase + g1 + (st - 3), seg[ph + uint32_t(g1 - d0) + (st - 3)]);
-                } else {
-                    named_bar_sync(2, kST);
-                    if (uint32_t(st) < A) stg_stream(p.tbase + d0 + st, seg[ph + st]);  // A < 8
+            } else if (PART) {
+                // Partition: trues at seg[0, A), falses at seg[A, A + F).  The trues'
+                // re-phase writes whole 16-byte chunks, up to seg[A + 6), so the
+                // first 7 falses are kept in registers until the trues' bulk store
+                // has read the stage.
+                const uint32_t F = uint32_t(ve0 - vs0) - A;
+                const uint32_t keep7 = (uint32_t(st) < 7 && uint32_t(st) < F) ? seg[A + st] : 0u;
+                named_bar_sync(2, kST);
+                if (A > 0) bulk_segment(p.tbase, p.tlo + meta[o].excl, A, 0u);
+                named_bar_sync(2, kST);
+                if (st == 0) {
+                    bulk_commit();
+                    bulk_wait_read<0>();  // the trues have been read out of the stage
                 }
+                named_bar_sync(2, kST);
+                if (uint32_t(st) < 7 && uint32_t(st) < F) seg[A + st] = keep7;
+                named_bar_sync(2, kST);
+                if (F > 0) bulk_segment(p.fbase, p.flo + ((vs0 - p.lo) - meta[o].excl), F, A);
+            } else if (!identity && A > 0) {
+                bulk_segment(p.tbase, p.tlo + meta[o].excl, A, 0u);
             }
 #endif
             named_bar_sync(2, kST);  // every storer is done reading the stage
