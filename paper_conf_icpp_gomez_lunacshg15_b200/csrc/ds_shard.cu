@@ -38,12 +38,39 @@ __global__ void shard_offsets_kernel(const uint64_t* counts, uint32_t world, uin
 // Grid-stride, one word per thread per iteration (coalesced on both sides).
 __global__ void tail_copy_kernel(uint32_t* dst_base, const uint64_t* d_offset, const uint32_t* src,
                                  uint64_t n_total) {
+    // Partition's second step: the falses, in order, from aux to ptr[off, n).
+    // Destination-aligned 16-byte stores; the source is read as 4 coalesced
+    // words per chunk (its phase relative to the destination is arbitrary).
     const uint64_t off = *d_offset;
     const uint64_t cnt = n_total - off;
     uint32_t* dst = dst_base + off;
-    for (uint64_t j = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; j < cnt;
-         j += uint64_t(gridDim.x) * blockDim.x)
-        dst[j] = src[j];
+    uint64_t head = (4u - uint32_t(reinterpret_cast<uintptr_t>(dst) >> 2)) & 3u;
+    if (head > cnt) head = cnt;
+    const uint64_t tid = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x;
+    const uint64_t nth = uint64_t(gridDim.x) * blockDim.x;
+    if (tid < head) dst[tid] = src[tid];
+    const uint64_t nchunks = (cnt - head) >> 2;
+    uint4* d4 = reinterpret_cast<uint4*>(dst + head);
+    const uint32_t* s4 = src + head;
+    constexpr int kU = 4;
+    for (uint64_t c0 = tid; c0 < nchunks; c0 += kU * nth) {
+        uint4 v[kU];
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const uint64_t c = c0 + u * nth;
+            if (c < nchunks) {
+                const uint32_t* q = s4 + 4 * c;
+                v[u] = make_uint4(__ldg(q), __ldg(q + 1), __ldg(q + 2), __ldg(q + 3));
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < kU; ++u) {
+            const uint64_t c = c0 + u * nth;
+            if (c < nchunks) d4[c] = v[u];
+        }
+    }
+    const uint64_t rest = head + 4 * nchunks;
+    if (tid < cnt - rest) dst[rest + tid] = src[rest + tid];
 }
 
 }  // namespace
