@@ -747,12 +747,15 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 const uint32_t mk = kMaskRegs ? mkr[c] : __shfl_sync(kFull, mymask, c);
                 if constexpr (kRc) r = wbase + rc[c];
                 const uint32_t rl = r + __popc(mk & lt);  // trues before this word in the tile
-                if (mk >> lane & 1u) {
-                    out[rl] = v[c];
-                } else if (PART) {
+                if constexpr (PART) {
+                    // one (predicated) shared store per word: true -> rank, false -> after the trues
                     const uint32_t x = uint32_t(xs + 32 * c + lane);
+                    const bool kb = mk >> lane & 1u;
+                    const uint32_t idx = kb ? rl : total + (x - vstart) - rl;
                     const uint64_t e = tb + x;
-                    if (e >= p.lo && e < p.hi) out[total + (x - vstart) - rl] = v[c];
+                    if (kb || (!guarded || (e >= p.lo && e < p.hi))) out[idx] = v[c];
+                } else if (mk >> lane & 1u) {
+                    out[rl] = v[c];
                 }
                 if constexpr (!kRc) r += __popc(mk);
             }
