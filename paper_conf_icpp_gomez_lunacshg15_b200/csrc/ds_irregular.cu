@@ -3,42 +3,40 @@
 // §III-B; primitives §IV-B/C P:230-282).
 //
 // One persistent, warp-specialised CTA per SM walks input tiles of
-// T = 8192 words in dynamic-ticket order (Fig. 4) through a 6-stage ring of
-// shared-memory tiles.  Each role works on a different tile at a time:
+// T = 8192 words in dynamic-ticket order (Fig. 4) through 4 input stages and
+// an output ring in shared memory.  Each role works on a different tile:
 //
-//   producer warp    a1 draws the next ticket as soon as a stage is free and
-//                    a2 loads the tile (plus, for unique, the 16 bytes before
-//                       it) with one TMA bulk copy (Alg. 2 lines 1-11; P:84
-//                       "on-chip memory")
-//  16 ranker warps   a3 keep flags (predicate / unique stencil), one
-//                       ballot per 32-word chunk (lane l holds word 32c + l)
-//                    a4 the tile aggregate ("Reduction") -- published
-//                       as AGG at once
-//                    a6 rank of every kept word in input order ("binary
-//                       prefix sum": popc of the chunk ballot
-//                       below the lane + a scan of the 16 warp totals); the
-//                       kept words are compacted in place, 32 consecutive
-//                       words per store
-//   6 resolver warps a5 (one per stage) decoupled look-back over 32
-//                       predecessors per round trip, started as soon as the
-//                       ticket is drawn (it needs no data), then INCL; the last
-//                       tile writes out_n (a8).  This replaces the serial flag
-//                       chain of Fig. 7, which is latency-bound on B200
-//
-//   5 storer warps   a7 re-phase the compacted words in shared memory to the
-//                       destination's 16-byte phase, one TMA bulk store of
-//                       [excl, excl + A) (scalar head/tail), then free the
-//                       stage once the bulk engine has read it
+//   producer warp    a1 draws the next ticket as soon as an input stage and a
+//                       slot are free; a2 loads the tile (plus, for unique,
+//                       the words before it) with one TMA bulk copy (Alg. 2
+//                       lines 1-11; "on-chip memory")
+//  16 ranker warps   a3 keep flags (predicate / unique stencil), 4 bits
+//                       per lane and 128-bit shared load; a4 the tile aggregate
+//                       ("Reduction"), published as AGG at once; the
+//                       input stage is released as soon as every ranker holds
+//                       its words in registers; a6 rank of every kept word in
+//                       input order ("binary prefix sum": one
+//                       shuffle scan over packed per-lane counts) and the
+//                       compaction of the kept words into the output ring
+//   8 resolver warps a5 decoupled look-back over 32 predecessors per round
+//                       trip, started as soon as the ticket is drawn (it needs
+//                       no data), then INCL; the last tile writes out_n (a8).
+//                       This replaces the serial flag chain of Fig. 7, which is
+//                       latency-bound on B200
+//   5 storer warps   a7 re-phase the tile's ring region to the destination's
+//                       16-byte phase, one TMA bulk store of [excl, excl + A)
+//                       (scalar head/tail), then free the region once the bulk
+//                       engine has read it
 //
 // A drawn tile's AGG depends only on its own load and ranking, never on the
-// resolution of earlier tiles.  In-place safety:
-// AGG/INCL are published only after the tile's copy completed; stores happen
-// only after the look-back saw AGG/INCL of every lower tile; outputs of tile t
-// lie in [0, (t+1)T), so no lower tile writes into a higher tile's input.
-// Deadlock freedom: look-backs wait only for lower (already drawn) tiles, and
-// a drawn tile reaches AGG without waiting on any other tile.
-#include <type_traits>
-
+// resolution of earlier tiles.  In-place safety: AGG/INCL
+// are published only after the tile's words were read out of the copy; stores
+// happen only after the look-back saw AGG/INCL of every lower tile; outputs
+// of tile t lie in [0, (t+1)T), so no lower tile writes into a higher tile's
+// input.  Deadlock freedom: look-backs wait only for lower (already drawn)
+// tiles; a drawn tile reaches AGG without waiting on any other tile; a ranker
+// waiting for ring space waits only for this CTA's lower tiles, whose
+// aggregates (and so all their predecessors' statuses) are already out.
 #include "ds_device.cuh"
 #include "ds_internal.h"
 
@@ -115,90 +113,117 @@ struct OpUnique64 {
     static constexpr bool kUnique = true, kWide = true;
 };
 
-__device__ __forceinline__ uint32_t lanemask_lt() {
-    uint32_t m;
-    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
-    return m;
-}
-
 // ---- CTA shape ----------------------------------------------------------
-#ifndef DS_IRR_RANK_WARPS
-#define DS_IRR_RANK_WARPS 16
-#endif
+// warps: 16 rankers (2 groups of 8) | 4 resolvers | 4 storers | 1 producer
 #ifndef DS_IRR_IN_STAGES
-#define DS_IRR_IN_STAGES 6
+#define DS_IRR_IN_STAGES 4
 #endif
 #ifndef DS_IRR_SLOTS
-#define DS_IRR_SLOTS 12
+#define DS_IRR_SLOTS 16
 #endif
 #ifndef DS_IRR_RESOLVERS
-#define DS_IRR_RESOLVERS 6
+#define DS_IRR_RESOLVERS 4
 #endif
-#ifndef DS_IRR_RANK_GROUPS
-#define DS_IRR_RANK_GROUPS 1
-#endif
-#ifndef DS_IRR_TILE
-#define DS_IRR_TILE 8192
-#endif
-constexpr int kRankWarps = DS_IRR_RANK_WARPS;
-constexpr int kRankGroups = DS_IRR_RANK_GROUPS;   // ranker groups, each on its own tile
-constexpr int kGroupWarps = kRankWarps / kRankGroups;
-constexpr int kRT = 32 * kGroupWarps;     // threads of one ranker group
-constexpr int kT = DS_IRR_TILE;           // words per tile (8192 = 32 KB)
-constexpr int kSeg = kT / kGroupWarps;    // contiguous words ranked by one warp (1024)
-constexpr int kChunks = kSeg / 32;        // 32-word chunks per warp segment (32)
-static_assert(kRankWarps % kRankGroups == 0 && kT % (32 * kGroupWarps) == 0, "ranker shape");
-static_assert(kChunks <= 32, "chunk masks are held one per lane");
-static_assert(kRankGroups <= 2, "named barriers 1 and 3 serve the ranker groups");
-constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
-constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
-constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
 #ifndef DS_IRR_STORE_WARPS
-#define DS_IRR_STORE_WARPS 5
+#define DS_IRR_STORE_WARPS 4
 #endif
-constexpr int kStoreWarps = DS_IRR_STORE_WARPS;
 #ifndef DS_IRR_BULK_STORE
 #define DS_IRR_BULK_STORE 1
 #endif
-constexpr bool kBulkStore = DS_IRR_BULK_STORE;  // a7 through TMA bulk stores (else 128-bit STG)
+constexpr bool kBulkStore = DS_IRR_BULK_STORE;  // a7 through TMA bulk stores (else 128-bit STG from registers)
+#ifndef DS_IRR_RANK_GROUPS
+#define DS_IRR_RANK_GROUPS 2
+#endif
+constexpr int kRankWarps = 16;
+constexpr int kRankGroups = DS_IRR_RANK_GROUPS;   // ranker groups, each on its own tile
+constexpr int kGroupWarps = kRankWarps / kRankGroups;
+constexpr int kRT = 32 * kGroupWarps;     // threads of one ranker group
+constexpr int kT = 8192;                  // words per tile (32 KB)
+constexpr int kSeg = kT / kGroupWarps;    // contiguous words ranked by one warp
+constexpr int kRounds = kSeg / 128;       // rounds of 4 words per lane
+constexpr int kPacks = (kRounds + 3) / 4; // registers of packed 8-bit round counts
+static_assert(kRankGroups == 1 || kRankGroups == 2, "named barriers 1 and 3 serve the ranker groups");
+static_assert(kRounds % 4 == 0, "whole packs of rounds");
+constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
+constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
+constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
+constexpr int kStoreWarps = DS_IRR_STORE_WARPS;
 constexpr int kST = 32 * kStoreWarps;
 constexpr int kWarpResolver0 = kRankWarps;
 constexpr int kWarpStorer0 = kRankWarps + kResolvers;
 constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;
 constexpr int kThreads = 32 * (kWarpProducer + 1);
-#ifndef DS_IRR_PRE
-#define DS_IRR_PRE 32
-#endif
-// Words before the tile in a stage (unique's boundary word).  Stages, and the
+// Words before the tile in a stage (unique's boundary words).  Stages, and the
 // tile inside each stage, start on 128-byte boundaries, so a bulk copy fills
 // whole 128-byte shared-memory lines and unique's copy (which starts kPre
 // words early) keeps a 128-byte aligned global source.
-constexpr int kPre = DS_IRR_PRE;
-#ifndef DS_IRR_ALIGN
-#define DS_IRR_ALIGN 32
+constexpr int kPre = 32;
+constexpr int kStageWords = kT + kPre + 32;
+// Output ring: the rankers compact each tile out of its input stage into the
+// ring (the stage is free as soon as every ranker holds its words in
+// registers); the storers drain the ring in tile order once the prefix is
+// known.  Everything left of the 227 KB after the input stages.
+constexpr int kStaticSmem = 2560;  // barriers, slot metadata (static shared memory; ptxas reports 2176 B)
+#ifndef DS_IRR_RING_WORDS
+#define DS_IRR_RING_WORDS (((227 * 1024 - kStaticSmem - 128) / 4 - kInStages * kStageWords) / 32 * 32)
 #endif
-constexpr int kAlignW = DS_IRR_ALIGN;    // stage alignment in words (32 = 128 bytes)
-constexpr int kStageWords = (kT + kPre + 4 + kAlignW - 1) / kAlignW * kAlignW;
-constexpr size_t kSmem = size_t(kInStages) * kStageWords * 4 + 128;  // + runtime alignment slack
-static_assert(kPre % 4 == 0 && kPre >= 4, "boundary words keep 16-byte alignment");
-static_assert(!DS_IRR_BULK_STORE || kStageWords >= kT + kPre + 8,
-              "re-phase writes whole chunks up to 6 words past a segment");
+constexpr int kRingWords = DS_IRR_RING_WORDS;
+constexpr size_t kSmem = (size_t(kInStages) * kStageWords + kRingWords) * 4 + 128;  // + alignment slack
+// A ring region is one tile's kept words (+ its false words for partition),
+// each rounded up to 4 words with 8 words of re-phase slack; a tile whose
+// region does not fit (now) is compacted in place instead.
+static_assert(kRingWords >= 0 && kRingWords % 4 == 0, "ring");
 static_assert(kThreads <= 1024, "CTA size");
 static_assert(kSlots >= kInStages, "a slot per input stage at least");
 static_assert(kSlots % kResolvers == 0, "a slot is always served by the same resolver");
-// 227 KB dynamic + static per CTA (the static part -- barriers, slot metadata --
-// is < 2.5 KB)
-static_assert(kSmem <= 227 * 1024 - 2560, "shared memory");
+static_assert(kSmem + kStaticSmem <= 227 * 1024, "shared memory");
 
 struct SlotMeta {
     uint32_t tile;              // kNoTile: end of this CTA's work
-    uint32_t prev_tile;         // this CTA's previous ticket (kNoTile: none)
-    volatile uint32_t incl_tile;          // == tile once incl is valid (CTA-local chain)
-    volatile unsigned long long incl;     // inclusive prefix of the tile
+    uint32_t stage;             // input stage holding the tile
     uint32_t total;             // kept words in the tile
+    uint32_t freed_snap;        // ring words freed when the tile was counted
     unsigned long long excl;    // kept words in all lower tiles
-    uint32_t wtot[kGroupWarps];  // kept words in each ranker warp's segment
+    uint32_t ring_pos;          // ring word of the tile's rank 0 (multiple of 4), or kNoTile: in its stage
+    uint32_t ring_end;          // ring allocation counter after this tile's decision (monotone)
+    uint32_t ring_hpos;         // ring position after this tile's decision
+    uint32_t wtot[kGroupWarps]; // kept words in each ranker warp's segment
 };
+
+__device__ __forceinline__ uint32_t round4(uint32_t x) { return (x + 3u) & ~3u; }
+// ring words a tile occupies: kept words (+ false words, partition)
+__device__ __forceinline__ uint32_t region_true(uint32_t total) { return total ? round4(total + 8u) : 0u; }
+__device__ __forceinline__ uint32_t region_false(uint32_t falses) { return falses ? round4(falses + 8u) : 0u; }
+
+__device__ __forceinline__ u32x4 lds_v4(uint32_t addr) {
+    u32x4 r;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "r"(addr));
+    return r;
+}
+__device__ __forceinline__ uint32_t lds_u32(uint32_t addr) {
+    uint32_t r;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(r) : "r"(addr));
+    return r;
+}
+__device__ __forceinline__ void sts_u32(uint32_t addr, uint32_t v) {
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
+}
+// The ring's free counter: storer -> rankers, ordered at CTA scope (the
+// storer's bulk reads of the freed words completed before its release).
+__device__ __forceinline__ void st_release_cta_smem(uint32_t* p, uint32_t v) {
+    asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_addr(p)), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire_cta_smem(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_addr(p)) : "memory");
+    return v;
+}
+// Free input stages (bit s): released (or) by the ranker / storer that is done
+// reading the stage, claimed (and-not) by the producer only.
+__device__ __forceinline__ void stage_release(uint32_t* mask, uint32_t s) {
+    asm volatile("atom.release.cta.shared::cta.or.b32 _, [%0], %1;" ::"r"(smem_addr(mask)), "r"(1u << s)
+                 : "memory");
+}
 
 // Shard halo (R18): last word of the nearest non-empty earlier shard.
 __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) {
@@ -212,227 +237,61 @@ __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) 
     return false;
 }
 
-// a5: decoupled look-back by one warp over 32 * kLB predecessors per round trip
-// (kLB = 1: fewer status sectors per poll beat a wider window).
-// Slot (m, lane) examines tile base - (32m + lane): every load instruction
-// reads 32 consecutive status words.  Waits only for the tiles up to the
-// nearest INCL predecessor.  Ends with one acquire fence per lane and a
-// __syncwarp so lane 0's later release is cumulative over all lanes.
-#ifndef DS_IRR_LB
-#define DS_IRR_LB 1
-#endif
-constexpr int kLB = DS_IRR_LB;  // look-back slots per lane (kLBW * kLB tiles per round)
-#ifndef DS_IRR_LBW
-#define DS_IRR_LBW 32
-#endif
-constexpr int kLBW = DS_IRR_LBW;  // lanes that read statuses (window width per slot row)
-static_assert(kLBW >= 1 && kLBW <= 32, "look-back lanes");
-#ifndef DS_IRR_REFRESH
-#define DS_IRR_REFRESH 1
-#endif
+// a5: decoupled look-back by one warp over 32 predecessors per round trip
+// (one sector per status; a wider window reads more sectors per poll, a
+// narrower one needs more round trips: DESIGN.md §7).  Lane l examines tile
+// base - l.  Waits only for the tiles up to the nearest INCL predecessor; the
+// nearest 32 AGG predecessors are re-read while polling (a nearer INCL ends
+// the walk sooner).  Ends with one acquire fence per lane (strict build) and
+// a __syncwarp so lane 0's later publication follows every lane's reads.
 #ifndef DS_IRR_POLL_MIN
 #define DS_IRR_POLL_MIN 64
 #endif
 #ifndef DS_IRR_POLL_MAX
 #define DS_IRR_POLL_MAX 512
 #endif
-constexpr int kRefreshRows = DS_IRR_REFRESH;        // AGG rows re-read while polling
 constexpr uint32_t kPollMinNs = DS_IRR_POLL_MIN;   // first back-off
 constexpr uint32_t kPollMaxNs = DS_IRR_POLL_MAX;   // back-off cap
-
-// Timing experiments only (wrong or unsafe results): DS_DEBUG_BISECT bits
-#ifndef DS_DEBUG_BISECT
-#define DS_DEBUG_BISECT 0
-#endif
-constexpr bool DBG_NO_PFENCE = DS_DEBUG_BISECT & 1, DBG_NO_PUBLISH = DS_DEBUG_BISECT & 2,
-               DBG_NO_BULKWAIT = DS_DEBUG_BISECT & 4, DBG_EARLY_FREE = DS_DEBUG_BISECT & 8,
-               DBG_SKIP_RANK = DS_DEBUG_BISECT & 16, DBG_NO_RFENCE = DS_DEBUG_BISECT & 32;
 #ifndef DS_IRR_LATE_LB
-#define DS_IRR_LATE_LB 0
+#define DS_IRR_LATE_LB 1
 #endif
-#ifndef DS_IRR_HELP
-#define DS_IRR_HELP 0
-#endif
-constexpr bool kHelp = DS_IRR_HELP;  // publish INCL for the nearest 32 AGG predecessors
-static_assert(!kHelp || kLBW == 32, "helper INCLs assume the 32-lane window");
+constexpr bool kLateLookback = DS_IRR_LATE_LB;
 
 __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint32_t tile,
                                              uint32_t epoch, int lane, uint64_t* trace) {
     uint64_t excl = 0;
     uint32_t rounds = 0, polls = 0;
     int64_t base = int64_t(tile) - 1;
-    uint64_t s0 = 0;     // the nearest 32 predecessors' statuses as the first round left them
-    uint32_t L0 = 32u;   // lanes of that row the walk needed (up to the nearest INCL)
+    uint32_t ns = kPollMinNs;
     while (true) {
-        uint64_t s[kLB];
-        uint32_t okm = 0;  // bit m: slot m holds a current status
-        const bool act = lane < kLBW;  // lanes of the window (the rest read as empty, current)
-#pragma unroll
-        for (int m = 0; m < kLB; ++m) {
-            const int64_t idx = base - (kLBW * m + lane);
-            s[m] = !act ? 0ull : idx >= 0 ? ld_relaxed_gpu(status_ptr(status, idx)) : make_status(kStateIncl, epoch, 0);
-        }
-#pragma unroll
-        for (int m = 0; m < kLB; ++m)
-            if (!act || status_current(s[m], epoch)) okm |= 1u << m;
+        int64_t idx = base - lane;
+        uint64_t s = idx >= 0 ? ld_relaxed_gpu(status_ptr(status, idx)) : make_status(kStateIncl, epoch, 0);
+        bool ok = status_current(s, epoch);
         if (rounds++ == 0 && lane == 0) trace_event(trace, tile, 10, globaltimer());
-        uint32_t ns = kPollMinNs;
-        uint32_t M, L;  // nearest INCL at slot M, lane L (M == kLB: none this round)
+        uint32_t L;  // nearest INCL at lane L (32: none this round)
         while (true) {
-            uint32_t inclm = 0;
-#pragma unroll
-            for (int m = 0; m < kLB; ++m)
-                if ((okm >> m & 1u) && status_state(s[m]) == kStateIncl) inclm |= 1u << m;
-            M = __reduce_min_sync(kFull, inclm ? uint32_t(__ffs(inclm) - 1) : uint32_t(kLB));
-            L = M < kLB ? uint32_t(__ffs(__ballot_sync(kFull, inclm >> M & 1u)) - 1) : 32u;
-            // needed: every slot before (M, L) in distance order, and (M, L)
-            const uint32_t need = (M < kLB ? ((1u << M) - 1u) : ((1u << kLB) - 1u)) |
-                                  (M < kLB && uint32_t(lane) <= L ? (1u << M) : 0u);
-            if (!__any_sync(kFull, (okm & need) != need)) break;
+            const uint32_t inclm = __ballot_sync(kFull, ok && status_state(s) == kStateIncl);
+            L = inclm ? uint32_t(__ffs(inclm) - 1) : 32u;
+            const bool need = uint32_t(lane) <= L;  // every lane up to the nearest INCL
+            if (!__any_sync(kFull, need && !ok)) break;
             __nanosleep(ns);
             ns = ns < kPollMaxNs ? ns * 2 : kPollMaxNs;
             ++polls;
-            // Re-read the needed slots that are still pending, and refresh the
-            // nearest 32 predecessors even if they hold AGG: a nearer INCL ends the
-            // walk sooner.  Farther AGG slots are not re-read (poll traffic hits
-            // the same few L2 lines from every resolver).
-#pragma unroll
-            for (int m = 0; m < kLB; ++m) {
-                const bool pending = !(okm >> m & 1u);
-                const bool refresh = act && m < kRefreshRows && !pending && status_state(s[m]) != kStateIncl;
-                if ((need >> m & 1u) && (pending || refresh)) {
-                    const int64_t idx = base - (kLBW * m + lane);
-                    if (idx >= 0) {
-                        s[m] = ld_relaxed_gpu(status_ptr(status, idx));
-                        okm = status_current(s[m], epoch) ? (okm | 1u << m) : (okm & ~(1u << m));
-                    }
-                }
+            if (need && (!ok || status_state(s) != kStateIncl) && idx >= 0) {
+                s = ld_relaxed_gpu(status_ptr(status, idx));
+                ok = status_current(s, epoch);
             }
         }
-        uint32_t agg = 0;
-        uint64_t inc = 0;
-#pragma unroll
-        for (int m = 0; m < kLB; ++m) {
-            if (uint32_t(m) < M || (uint32_t(m) == M && uint32_t(lane) < L)) agg += uint32_t(status_count(s[m]));
-            if (uint32_t(m) == M && uint32_t(lane) == L) inc = status_count(s[m]);
-        }
+        const uint32_t agg = uint32_t(lane) < L ? uint32_t(status_count(s)) : 0u;
         excl += uint64_t(__reduce_add_sync(kFull, agg));
-        if (rounds == 1) {
-            s0 = s[0];
-            L0 = M == 0 ? L : 32u;
-        }
-        if (M < kLB) {
-            excl += __shfl_sync(kFull, inc, L);
+        if (L < 32u) {
+            excl += __shfl_sync(kFull, status_count(s), L);
             break;
         }
-        base -= kLBW * kLB;
-    }
-    if (kHelp) {
-        // The walk fixed the inclusive prefix of every tile it summed: for the
-        // nearest predecessors t-1-l (l < L0, all AGG), incl = excl - (counts of
-        // t-1 .. t-l).  Publishing them lets later look-backs stop sooner.  A
-        // racing writer (the tile's own resolver, another helper) stores the
-        // same word.
-        const uint32_t c0 = uint32_t(lane) < L0 ? uint32_t(status_count(s0)) : 0u;
-        uint32_t pre = c0;
-#pragma unroll
-        for (int sh = 1; sh < 32; sh <<= 1) {
-            const uint32_t y = __shfl_up_sync(kFull, pre, sh);
-            if (lane >= sh) pre += y;
-        }
-        pre -= c0;  // exclusive: counts of the lanes nearer than this one
-        const int64_t idx = int64_t(tile) - 1 - lane;
-        if (uint32_t(lane) < L0 && idx >= 0 && status_state(s0) == kStateAgg)
-            publish_status(status_ptr(status, idx), make_status(kStateIncl, epoch, excl - pre));
+        base -= 32;
     }
     if (lane == 0) {
         trace_event(trace, tile, 8, rounds);
-        trace_event(trace, tile, 9, polls);
-        trace_event(trace, tile, 11, globaltimer());
-    }
-    lookback_acquire();
-    __syncwarp();
-    if (lane == 0) trace_event(trace, tile, 12, globaltimer());
-    return excl;
-}
-
-#ifndef DS_IRR_LOCAL_CHAIN
-#define DS_IRR_LOCAL_CHAIN 0
-#endif
-constexpr bool kLocalChain = DS_IRR_LOCAL_CHAIN;
-#ifndef DS_IRR_LW
-#define DS_IRR_LW 8
-#endif
-constexpr int kLW = DS_IRR_LW;  // window slots per lane (32 * kLW tiles)
-
-// a5, CTA-local chain: this CTA's previous tile tp < t resolves first (its
-// resolver is in the same CTA), so t needs only the aggregates of the window
-// (tp, t) -- about one tile per other SM -- plus incl(tp) from shared memory,
-// or a nearer INCL inside the window.  One read of the window (<= 32*kLB
-// tiles), then only its pending slots are re-read; no multi-round walk.
-__device__ __forceinline__ uint64_t lookback_window(const uint64_t* __restrict__ status, uint32_t tile,
-                                                    uint32_t tp, const SlotMeta* pm, uint32_t epoch,
-                                                    int lane, uint64_t* trace) {
-    const uint32_t W = tile - tp - 1;  // window tiles tile-1 .. tp+1
-    const int64_t base = int64_t(tile) - 1;
-    uint64_t s[kLW];
-    uint32_t okm = 0;  // bit m: slot m current (or outside the window)
-#pragma unroll
-    for (int m = 0; m < kLW; ++m) {
-        const uint32_t d = uint32_t(32 * m + lane);
-        if (d < W) {
-            s[m] = ld_relaxed_gpu(status_ptr(status, base - d));
-            if (status_current(s[m], epoch)) okm |= 1u << m;
-        } else {
-            s[m] = 0;
-            okm |= 1u << m;
-        }
-    }
-    if (lane == 0) trace_event(trace, tile, 10, globaltimer());
-    uint32_t ns = kPollMinNs, polls = 0;
-    uint32_t M, L;
-    bool local;
-    while (true) {
-        uint32_t inclm = 0;
-#pragma unroll
-        for (int m = 0; m < kLW; ++m)
-            if (uint32_t(32 * m + lane) < W && (okm >> m & 1u) && status_state(s[m]) == kStateIncl) inclm |= 1u << m;
-        M = __reduce_min_sync(kFull, inclm ? uint32_t(__ffs(inclm) - 1) : uint32_t(kLW));
-        L = M < kLW ? uint32_t(__ffs(__ballot_sync(kFull, inclm >> M & 1u)) - 1) : 32u;
-        const uint32_t need = (M < kLW ? ((1u << M) - 1u) : ((1u << kLW) - 1u)) |
-                              (M < kLW && uint32_t(lane) <= L ? (1u << M) : 0u);
-        const bool have = !__any_sync(kFull, (okm & need) != need);
-        local = M == kLW && __shfl_sync(kFull, pm->incl_tile, 0) == tp;
-        if (have && (M < kLW || local)) break;
-        __nanosleep(ns);
-        ns = ns < kPollMaxNs ? ns * 2 : kPollMaxNs;
-        ++polls;
-#pragma unroll
-        for (int m = 0; m < kLW; ++m) {
-            const bool pending = !(okm >> m & 1u);
-            const bool refresh = m < kRefreshRows && !pending && status_state(s[m]) != kStateIncl;
-            if ((need >> m & 1u) && (pending || (refresh && !local))) {
-                const int64_t idx = base - (32 * m + lane);
-                if (uint32_t(32 * m + lane) < W) {
-                    s[m] = ld_relaxed_gpu(status_ptr(status, idx));
-                    okm = status_current(s[m], epoch) ? (okm | 1u << m) : (okm & ~(1u << m));
-                }
-            }
-        }
-    }
-    uint32_t agg = 0;
-    uint64_t inc = 0;
-#pragma unroll
-    for (int m = 0; m < kLW; ++m) {
-        const bool inw = uint32_t(32 * m + lane) < W;
-        if (inw && (uint32_t(m) < M || (uint32_t(m) == M && uint32_t(lane) < L))) agg += uint32_t(status_count(s[m]));
-        if (uint32_t(m) == M && uint32_t(lane) == L) inc = status_count(s[m]);
-    }
-    uint64_t excl = uint64_t(__reduce_add_sync(kFull, agg));
-    __threadfence_block();  // incl was written before incl_tile
-    excl += M < kLW ? __shfl_sync(kFull, inc, L) : pm->incl;
-    if (lane == 0) {
-        trace_event(trace, tile, 8, M < kLW ? 1 : 0);
         trace_event(trace, tile, 9, polls);
         trace_event(trace, tile, 11, globaltimer());
     }
@@ -494,7 +353,7 @@ __device__ __forceinline__ void store_segment(uint32_t* base, uint64_t d0, uint3
 
 // a7 helper: move the cnt words seg[0, cnt) to seg[ph, ph + cnt) in shared
 // memory (ph = 1..3; seg 16-byte aligned with >= 4 readable words before it
-// and >= 4 writable words after the segment).  Destination chunk c (words
+// and >= 6 writable words after the segment).  Destination chunk c (words
 // [4c, 4c+4)) takes source words [4c-ph, 4c+4-ph): two aligned vector loads.
 // Writing chunk c destroys sources of chunk c+1 only, so the chunks go in
 // descending rounds, each reading everything before writing.
@@ -528,18 +387,21 @@ __device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph
     }
 }
 
-
 // mbarrier wait that also returns (false) once the CTA's work is known to
-// end before ring position k (the resolvers take alternate positions, so the
-// one not holding the end marker is released this way).
+// end before ring position k (the resolvers take every kResolvers-th
+// position, so the ones not holding the end marker are released this way).
 // Suspend-time hint of those waits: it bounds how long a warp parked on a
 // position past the end keeps the CTA (and so the launch) alive.
 #ifndef DS_IRR_END_POLL_NS
 #define DS_IRR_END_POLL_NS 1000
 #endif
 constexpr uint32_t kEndPollNs = DS_IRR_END_POLL_NS;
+#ifndef DS_IRR_TESTWAIT
+#define DS_IRR_TESTWAIT 1
+#endif
 __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
                                                  const volatile uint32_t* s_end, uint32_t k) {
+    if (DS_IRR_TESTWAIT && mbar_test_wait(bar, parity)) return true;  // no suspension if already complete
     while (true) {
         if (mbar_try_wait(bar, parity, kEndPollNs)) return true;
         // Strictly beyond the end marker: the position holding the marker
@@ -548,26 +410,53 @@ __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
     }
 }
 
+// a3: keep bits of the 4 words a lane holds in one round (bit j = word
+// x0 + j), for 4-byte words.  pw = the word before x0 (unique).
+template <class Op>
+__device__ __forceinline__ uint32_t keep_bits4(const u32x4& v, uint32_t pw, uint32_t value) {
+    if constexpr (Op::kUnique) {
+        return uint32_t(v.x != pw) | uint32_t(v.y != v.x) << 1 | uint32_t(v.z != v.y) << 2 |
+               uint32_t(v.w != v.z) << 3;
+    } else {
+        return uint32_t(Op::keep(v.x, value)) | uint32_t(Op::keep(v.y, value)) << 1 |
+               uint32_t(Op::keep(v.z, value)) << 2 | uint32_t(Op::keep(v.w, value)) << 3;
+    }
+}
+// Same for 8-byte elements (x, y) and (z, w): both words of an element get its
+// flag.  (pz, pw) = the element before (x, y) (unique).
+template <class Op>
+__device__ __forceinline__ uint32_t keep_bits4_wide(const u32x4& v, uint32_t pz, uint32_t pw, uint64_t value) {
+    bool k0, k1;
+    if constexpr (Op::kUnique) {
+        k0 = v.x != pz || v.y != pw;
+        k1 = v.z != v.x || v.w != v.y;
+    } else {
+        k0 = Op::keep2(uint64_t(v.y) << 32 | v.x, value);
+        k1 = Op::keep2(uint64_t(v.w) << 32 | v.z, value);
+    }
+    return (k0 ? 3u : 0u) | (k1 ? 12u : 0u);
+}
+
 template <class Op, bool PART>
 __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParams p) {
     extern __shared__ __align__(128) uint32_t smem_raw[];
     // 128-byte aligned stage base (offset arithmetic keeps the shared window,
     // so the stage accesses stay LDS/STS)
     uint32_t* const smem = smem_raw + ((128u - (smem_addr(smem_raw) & 127u)) & 127u) / 4u;
-    __shared__ __align__(8) uint64_t bar_full[kInStages], bar_free[kInStages];
-    __shared__ __align__(8) uint64_t bar_drawn[kSlots], bar_counted[kSlots], bar_ranked[kSlots],
-        bar_resolved[kSlots], bar_stored[kSlots];
+    uint32_t* const ring = smem + kInStages * kStageWords;
+    __shared__ __align__(8) uint64_t bar_loaded[kSlots], bar_drawn[kSlots], bar_counted[kSlots],
+        bar_ranked[kSlots], bar_resolved[kSlots], bar_stored[kSlots];
     __shared__ SlotMeta meta[kSlots];
     __shared__ uint32_t s_epoch;
-    __shared__ volatile uint32_t s_end;        // ring position of the end marker
+    __shared__ volatile uint32_t s_end;  // ring position of the end marker
+    __shared__ uint32_t s_freed;         // output-ring words released by the storers (monotone)
+    __shared__ uint32_t s_stages;        // free input stages (bit mask)
+    __shared__ uint32_t s_alloc;         // ring positions whose ring decision is out
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
-        for (int s = 0; s < kInStages; ++s) {
-            mbar_init(&bar_full[s], 1);
-            mbar_init(&bar_free[s], 1);
-        }
         for (int o = 0; o < kSlots; ++o) {
+            mbar_init(&bar_loaded[o], 1);
             mbar_init(&bar_drawn[o], 1);
             mbar_init(&bar_counted[o], 1);
             mbar_init(&bar_ranked[o], kGroupWarps);
@@ -575,6 +464,9 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             mbar_init(&bar_stored[o], 1);
         }
         s_end = 0xffffffffu;
+        s_freed = 0;
+        s_stages = (1u << kInStages) - 1u;
+        s_alloc = 0;
         mbar_fence_init();
     }
     __syncthreads();
@@ -582,12 +474,16 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
     if (warp == kWarpProducer) {
         // ------------------------------------------------ producer (lane 0)
         if (lane != 0) return;
-        uint32_t prev_t = kNoTile;
         for (uint32_t k = 0;; ++k) {
-            const int s = k % kInStages, o = k % kSlots;
+            const int o = k % kSlots;
+            mbar_wait(&bar_stored[o], ((k / kSlots) & 1) ^ 1);  // slot o finished tile k - kSlots
+            // any free input stage (a tile compacted into the ring frees its stage at
+            // once, one compacted in place only once stored)
+            uint32_t m;
+            while ((m = ld_acquire_cta_smem(&s_stages)) == 0u) __nanosleep(32);
+            const uint32_t s = __ffs(m) - 1;
+            atomicAnd(&s_stages, ~(1u << s));
             uint32_t* stage = smem + s * kStageWords;
-            mbar_wait(&bar_free[s], ((k / kInStages) & 1) ^ 1);  // rankers hold tile k - kInStages
-            mbar_wait(&bar_stored[o], ((k / kSlots) & 1) ^ 1);   // slot o finished tile k - kSlots
             uint32_t t, epoch;
             draw_ticket(p.ctrl, p.draws, t, epoch);
             if (k == 0) s_epoch = epoch;
@@ -595,126 +491,168 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 meta[o].tile = kNoTile;
                 s_end = k;
                 mbar_arrive(&bar_drawn[o]);
-                mbar_arrive(&bar_full[s]);
+                mbar_arrive(&bar_loaded[o]);
+                // End markers for the other resolvers' next positions, so each of
+                // them finds one and no warp has to poll for the end of the work.
+                for (uint32_t j = 1; j < uint32_t(kResolvers); ++j) {
+                    const uint32_t kj = k + j, oj = kj % kSlots;
+                    mbar_wait(&bar_stored[oj], ((kj / kSlots) & 1) ^ 1);
+                    meta[oj].tile = kNoTile;
+                    mbar_arrive(&bar_drawn[oj]);
+                }
                 return;
             }
             meta[o].tile = t;
-            meta[o].prev_tile = prev_t;
-            prev_t = t;
+            meta[o].stage = s;
             mbar_arrive(&bar_drawn[o]);  // the resolver starts this tile's look-back now
             trace_event(p.trace, t, 0, globaltimer());
             trace_event(p.trace, t, 7, smid());
             debug_delay(t, 0);
             const uint64_t tb = uint64_t(t) * kT;
             uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
-            end = (end + 3) & ~3ull;  // may read <= 12 bytes past the array end (same 16 B chunk)
-            // Unique also needs the word before the tile: one copy starting 16
-            // bytes early (measured faster than a separate 16-byte copy).
+            // The copy covers whole 16-byte chunks: it may read up to 12 bytes past
+            // the array end and the (lo) words before ptr, inside the same chunks
+            // (include/ds.h, "Reads").
+            end = (end + 3) & ~3ull;
+            // Unique also needs the word before the tile: one copy starting kPre
+            // words early (measured faster than a separate 16-byte copy).
             const uint64_t beg = (Op::kUnique && t > 0) ? tb - kPre : tb;
             const uint32_t bytes = uint32_t(end - beg) * 4u;
-            if (!DBG_NO_PFENCE) fence_proxy_async_smem();
-            mbar_arrive_expect_tx(&bar_full[s], bytes);
-            bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_full[s]);
+            fence_proxy_async_smem();
+            mbar_arrive_expect_tx(&bar_loaded[o], bytes);
+            bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_loaded[o]);
         }
     } else if (warp < kRankWarps) {
         // ------------------------------------------------ ranker warps
-        // kRankGroups groups of kGroupWarps warps; group g ranks the tiles at
-        // ring positions k = g (mod kRankGroups), so one group's barrier, scan
-        // and status store overlap the other group's loads and ballots.
+        // kRankGroups groups of kGroupWarps warps; group g ranks the tiles at ring
+        // positions k = g (mod kRankGroups), so one group's shuffle-scan chains and
+        // barrier overlap the other group's loads and stores.  Warp rw of a group
+        // ranks tile words [xs, xs + kSeg) in rounds of 128: in round r lane l
+        // holds the 4 words xs + 128r + 4l + {0..3} (one 128-bit shared load,
+        // conflict-free).  Keep flags are 4 bits per lane and round (a3), counted
+        // per lane; 4 rounds' counts travel in 8-bit fields of one register
+        // through ONE shuffle scan over the lanes, which gives every lane its
+        // exclusive offset in those rounds at once (a4/a6).  No ballot and no
+        // per-word POPC: those run at a quarter of the ALU rate and bound the
+        // chunked ballot ranker.
         const int g = warp / kGroupWarps, rw = warp % kGroupWarps;
-        const int rt = tid - g * kRT;  // thread index within the group
-        const uint32_t gbar = 1 + 2 * g;  // named barrier of the group (2 is the storers')
-        const uint32_t lt = lanemask_lt();
+        const int rt = tid - g * kRT;         // thread index within the group
+        const uint32_t gbar = 1 + 2 * g;      // named barrier of the group (2 is the storers')
+        const int xs = kSeg * rw;
+        const uint32_t smem_b = smem_addr(smem);
+        const uint32_t ring_b = smem_addr(ring);
         bool has_hprev = false;
         uint32_t hprev = 0;
-        if (Op::kUnique) has_hprev = halo_prev(p, hprev);
+        if (Op::kUnique && !Op::kWide) has_hprev = halo_prev(p, hprev);
         for (uint32_t k = g;; k += kRankGroups) {
-            const int s = k % kInStages, o = k % kSlots;
-            uint32_t* stage = smem + s * kStageWords;
-            // the other group's end position releases this group too
-            if (!mbar_wait_or_end(&bar_full[s], (k / kInStages) & 1, &s_end, k)) break;
+            const int o = k % kSlots;
+            if (!mbar_wait_or_end(&bar_loaded[o], (k / kSlots) & 1, &s_end, k)) break;
             const uint32_t t = meta[o].tile;
             if (t == kNoTile) break;
+            const uint32_t s = meta[o].stage;
             if (rt == 0) trace_event(p.trace, t, 1, globaltimer());
-            if (DBG_SKIP_RANK) {  // timing experiment only
-                named_bar_sync(gbar, kRT);
-                if (rt == 0) {
-                    meta[o].total = 0;
-                    publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, 0));
-                    mbar_arrive(&bar_counted[o]);
-                }
-                if (lane == 0) mbar_arrive(&bar_ranked[o]);
-                continue;
-            }
             const uint64_t tb = uint64_t(t) * kT;
             const bool full = tb >= p.lo && tb + kT <= p.hi;
-
-            // a3/a4: warp rw ranks tile words [xs, xs + kSeg) in kChunks chunks of
-            // 32: lane l holds word x = xs + 32c + l of chunk c, so every shared
-            // load and every compaction store below touches 32 consecutive words
-            // (no bank conflicts), and a chunk's keep flags are one ballot.  The
-            // ballot of chunk c is kept by lane c (one register instead of kChunks).
-            const int xs = kSeg * rw;
-            constexpr bool kMaskRegs = kChunks <= 16;  // else chunk c's mask is held by lane c
-            constexpr bool kRc = kMaskRegs && !PART;  // chunk offsets from the count (registers)
-            uint32_t v[kChunks];
-            uint32_t mkr[kMaskRegs ? kChunks : 1], rc[kRc ? kChunks : 1];
-            uint32_t mymask = 0;  // lane c: keep mask of chunk c (!kMaskRegs)
-            uint32_t wrun = 0;    // kept words of the warp's segment
-#pragma unroll
-            for (int c = 0; c < kChunks; ++c) v[c] = stage[kPre + xs + 32 * c + lane];
-            // Tile-relative bounds: only tile 0 (the array's first word, the lead
-            // words below p.lo) and the last tile need the guarded pass; every
-            // other tile takes the branch-free pass (same ops, no range checks).
+            // Tile-relative valid range: only tile 0 (lead words below p.lo) and the
+            // last tile need range checks.
             const uint32_t xlo = tb < p.lo ? uint32_t(p.lo - tb) : 0u;
             const uint32_t xhi = tb + kT <= p.hi ? uint32_t(kT) : uint32_t(p.hi - tb);
             const bool guarded = !full || t == 0;
-            auto count_pass = [&](auto guard_tag) {
-                constexpr bool G = decltype(guard_tag)::value;
+            const uint32_t st_b = smem_b + 4u * (s * uint32_t(kStageWords) + kPre);  // tile word 0
+            u32x4 v[kRounds];
 #pragma unroll
-                for (int c = 0; c < kChunks; ++c) {
-                    const uint32_t x = uint32_t(xs + 32 * c + lane);
-                    bool kp;
-                    if constexpr (Op::kWide) {
-                        // element = (even word, odd word) = lanes (2m, 2m+1) of the chunk
-                        const uint32_t partner = __shfl_xor_sync(kFull, v[c], 1);
-                        const uint32_t lo = (lane & 1) ? partner : v[c], hi = (lane & 1) ? v[c] : partner;
-                        const uint32_t xe = x - (lane & 1);  // the element's first word
-                        if constexpr (Op::kUnique) {
-                            kp = lo != stage[kPre + xe - 2] || hi != stage[kPre + xe - 1];
-                            if (G && t == 0 && xe == xlo) kp = true;  // the array's first element
-                        } else {
-                            kp = Op::keep2((uint64_t(hi) << 32) | lo, (uint64_t(p.value_hi) << 32) | p.value);
+            for (int r = 0; r < kRounds; ++r) v[r] = lds_v4(st_b + 4u * uint32_t(xs + 128 * r + 4 * lane));
+            uint32_t kb = 0, P[kPacks];
+#pragma unroll
+            for (int i = 0; i < kPacks; ++i) P[i] = 0;
+#pragma unroll
+            for (int r = 0; r < kRounds; ++r) {
+                const uint32_t x0 = uint32_t(xs + 128 * r + 4 * lane);
+                uint32_t b;
+                if constexpr (Op::kWide) {
+                    uint32_t pz = 0, pw = 0;
+                    if constexpr (Op::kUnique) {
+                        // element before (x, y): lane l-1's (z, w), lane 31 of the previous
+                        // round, or the two staged words before the segment
+                        pz = __shfl_up_sync(kFull, v[r].z, 1);
+                        pw = __shfl_up_sync(kFull, v[r].w, 1);
+                        if (r > 0) {
+                            const uint32_t lz = __shfl_sync(kFull, v[r > 0 ? r - 1 : 0].z, 31);
+                            const uint32_t lw = __shfl_sync(kFull, v[r > 0 ? r - 1 : 0].w, 31);
+                            if (lane == 0) pz = lz, pw = lw;
+                        } else if (lane == 0) {
+                            pz = lds_u32(st_b + 4u * uint32_t(xs - 2));
+                            pw = lds_u32(st_b + 4u * uint32_t(xs - 1));
                         }
-                    } else if constexpr (Op::kUnique) {
-                        // previous word straight from the staged tile; x == 0 reads
-                        // the word before the tile
-                        kp = v[c] != stage[kPre + x - 1];
-                        if (G && t == 0 && x == xlo) kp = !has_hprev || v[c] != hprev;  // the array's first word (R18)
-                    } else {
-                        kp = Op::keep(v[c], p.value);
                     }
-                    if (G) kp = kp && x >= xlo && x < xhi;
-                    const uint32_t mk = __ballot_sync(kFull, kp);
-                    if constexpr (kMaskRegs) {
-                        mkr[c] = mk;
-                        if constexpr (kRc) rc[c] = wrun;  // kept words of the segment before chunk c
-                    } else if (lane == c) {
-                        mymask = mk;
+                    b = keep_bits4_wide<Op>(v[r], pz, pw, uint64_t(p.value_hi) << 32 | p.value);
+                    if (Op::kUnique && guarded && t == 0) {  // the array's first element is kept
+                        if (x0 == xlo) b |= 3u;
+                        if (x0 + 2 == xlo) b |= 12u;
                     }
-                    wrun += __popc(mk);
+                } else {
+                    uint32_t pw = 0;
+                    if constexpr (Op::kUnique) {
+                        // word before x0: lane l-1's last word, lane 31 of the previous
+                        // round, or the staged word before the segment (P:280 for xs = 0)
+                        pw = __shfl_up_sync(kFull, v[r].w, 1);
+                        if (r > 0) {
+                            const uint32_t lw = __shfl_sync(kFull, v[r > 0 ? r - 1 : 0].w, 31);
+                            if (lane == 0) pw = lw;
+                        } else if (lane == 0) {
+                            pw = lds_u32(st_b + 4u * uint32_t(xs - 1));
+                        }
+                    }
+                    b = keep_bits4<Op>(v[r], pw, p.value);
+                    if (Op::kUnique && guarded && t == 0 && x0 <= xlo && xlo < x0 + 4) {
+                        // the array's first word (R18): kept unless it equals the halo word
+                        const uint32_t j = xlo - x0;
+                        const uint32_t w0 = j == 0 ? v[r].x : j == 1 ? v[r].y : j == 2 ? v[r].z : v[r].w;
+                        const bool k0 = !has_hprev || w0 != hprev;
+                        b = (b & ~(1u << j)) | (uint32_t(k0) << j);
+                    }
                 }
-            };
-            if (guarded) count_pass(std::true_type{});
-            else count_pass(std::false_type{});
+                if (guarded) {
+                    // words outside [xlo, xhi) are not elements of the array
+                    const uint32_t lo_ok = x0 >= xlo ? 15u : (15u << (xlo - x0)) & 15u;
+                    const uint32_t hi_ok = x0 + 4 <= xhi ? 15u : x0 >= xhi ? 0u : (1u << (xhi - x0)) - 1u;
+                    b &= lo_ok & hi_ok;
+                }
+                kb |= b << (4 * r);
+                P[r / 4] += uint32_t(__popc(b)) << (8 * (r % 4));
+            }
+            // exclusive offsets of every lane in all rounds (8-bit fields, <= 128 each)
+            uint32_t inc[kPacks];
+#pragma unroll
+            for (int i = 0; i < kPacks; ++i) inc[i] = P[i];
+#pragma unroll
+            for (int sh = 1; sh < 32; sh <<= 1) {
+#pragma unroll
+                for (int i = 0; i < kPacks; ++i) {
+                    const uint32_t y = __shfl_up_sync(kFull, inc[i], sh);
+                    if (lane >= sh) inc[i] += y;
+                }
+            }
+            uint32_t E[kPacks], R[kRounds];  // R[r]: kept words of the segment before round r
+            uint32_t wrun = 0;               // kept words of the warp's segment
+#pragma unroll
+            for (int i = 0; i < kPacks; ++i) {
+                E[i] = inc[i] - P[i];
+                const uint32_t T4 = __shfl_sync(kFull, inc[i], 31);
+#pragma unroll
+                for (int f = 0; f < 4; ++f) {
+                    R[4 * i + f] = wrun;
+                    wrun += T4 >> (8 * f) & 255u;
+                }
+            }
             if (lane == 0) meta[o].wtot[rw] = wrun;
-            if (rt == 0) trace_event(p.trace, t, 13, globaltimer());
+            if (rt == 0) {
+                meta[o].freed_snap = ld_acquire_cta_smem(&s_freed);  // one ring view for the group
+                trace_event(p.trace, t, 13, globaltimer());
+            }
             named_bar_sync(gbar, kRT);  // warp totals written; every ranker holds its words
-            if (DBG_EARLY_FREE && rt == 0) mbar_arrive(&bar_free[s]);  // timing experiment only
             if (rt == 0) trace_event(p.trace, t, 14, globaltimer());
-
-            // Exclusive scan of the group's warp totals (input order), redundantly
-            // in every warp.
+            // Exclusive scan of the warp totals (input order), redundantly in every warp.
             const uint32_t cw = lane < kGroupWarps ? meta[o].wtot[lane] : 0u;
             uint32_t iw = cw;
 #pragma unroll
@@ -729,37 +667,79 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 // (a relaxed status store).
                 meta[o].total = total;
                 debug_delay(t, 1);
-                if (!DBG_NO_PUBLISH) publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
+                publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
                 trace_event(p.trace, t, 2, globaltimer());
                 mbar_arrive(&bar_counted[o]);
             }
-
-            // a6: compact the kept words in place, rank r -> stage[kPre + r]
-            // (every ranker's words are in registers since the barrier).
-            // Partition also places the false words, in input order, after the
-            // trues: the f-th false word goes to stage[kPre + total + f], where
-            // f = (valid words before it in the tile) - (true words before it).
-            uint32_t* out = stage + kPre;
-            const uint32_t vstart = tb < p.lo ? uint32_t(p.lo - tb) : 0u;  // invalid lead words (tile 0)
-            uint32_t r = wbase;
-#pragma unroll
-            for (int c = 0; c < kChunks; ++c) {
-                const uint32_t mk = kMaskRegs ? mkr[c] : __shfl_sync(kFull, mymask, c);
-                if constexpr (kRc) r = wbase + rc[c];
-                const uint32_t rl = r + __popc(mk & lt);  // trues before this word in the tile
-                if constexpr (PART) {
-                    // one (predicated) shared store per word: true -> rank, false -> after the trues
-                    const uint32_t x = uint32_t(xs + 32 * c + lane);
-                    const bool kb = mk >> lane & 1u;
-                    const uint32_t idx = kb ? rl : total + (x - vstart) - rl;
-                    const uint64_t e = tb + x;
-                    if (kb || (!guarded || (e >= p.lo && e < p.hi))) out[idx] = v[c];
-                } else if (mk >> lane & 1u) {
-                    out[rl] = v[c];
+            // Where the compacted tile waits for its prefix: a region of the output
+            // ring if the ring has room (the input stage is then free at once), else
+            // in place in its input stage (held until stored).  Rankers never wait
+            // for ring space: a blocked ranker would keep drawn tiles from
+            // publishing their aggregates and stall every look-back behind them.
+            // Ring regions are allocated in ring-position order: position k starts
+            // from position k-1's allocation state (meta of the previous slot, valid
+            // once s_alloc reaches k); every thread of the group computes the same
+            // decision from the same snapshot.
+            uint32_t h = 0, hp = 0;
+            if (k > 0) {
+                if (kRankGroups > 1) {
+                    if (lane == 0)
+                        while (ld_acquire_cta_smem(&s_alloc) < k) __nanosleep(32);
+                    __syncwarp();
                 }
-                if constexpr (!kRc) r += __popc(mk);
+                const SlotMeta& pm = meta[(k + kSlots - 1) % kSlots];
+                h = pm.ring_end;
+                hp = pm.ring_hpos;
             }
-            if (!DBG_NO_RFENCE) fence_proxy_async_smem();  // the compacted words leave through a bulk store
+            const uint32_t falses = PART ? (xhi - xlo) - total : 0u;
+            const uint32_t need_t = region_true(total);
+            const uint32_t need = need_t + region_false(falses);
+            const uint32_t h0 = h, hp0 = hp;
+            if (hp + need > uint32_t(kRingWords)) {  // no wrapped regions: skip the ring's end
+                h += uint32_t(kRingWords) - hp;
+                hp = 0;
+            }
+            const bool in_ring = h + need - meta[o].freed_snap <= uint32_t(kRingWords);
+            const uint32_t rpos = hp;
+            if (rt == 0) {
+                meta[o].ring_pos = in_ring ? rpos : kNoTile;
+                meta[o].ring_end = in_ring ? h + need : h0;
+                meta[o].ring_hpos = in_ring ? hp + need : hp0;
+                if (kRankGroups > 1) st_release_cta_smem(&s_alloc, k + 1);
+                if (in_ring) stage_release(&s_stages, s);  // every ranker of the group holds its words
+            }
+            // a6: compact the kept words, rank r -> out[r] (partition: the f-th false
+            // word -> out[need_t + f]), out = ring + rpos or the tile's stage.
+            if (PART || wrun != 0) {
+                const uint32_t out_b = in_ring ? ring_b + 4u * rpos : st_b;
+#pragma unroll
+                for (int r = 0; r < kRounds; ++r) {
+                    const uint32_t b = kb >> (4 * r) & 15u;
+                    const uint32_t q0 = wbase + R[r] + (E[r / 4] >> (8 * (r % 4)) & 255u);  // trues before word x0
+                    const uint32_t q1 = q0 + (b & 1u), q2 = q1 + (b >> 1 & 1u), q3 = q2 + (b >> 2 & 1u);
+                    if constexpr (PART) {
+                        // one (predicated) shared store per valid word: true -> its rank,
+                        // false -> after the trues' region, in input order
+                        const uint32_t x0 = uint32_t(xs + 128 * r + 4 * lane);
+                        const uint32_t fb = need_t + x0 - xlo;  // + (valid words before x0) - trues before
+                        const uint32_t q[4] = {q0, q1, q2, q3};
+                        const uint32_t w[4] = {v[r].x, v[r].y, v[r].z, v[r].w};
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const uint32_t x = x0 + j;
+                            const bool kt = b >> j & 1u;
+                            const uint32_t idx = kt ? q[j] : fb + j - q[j];
+                            if (kt || !guarded || (x >= xlo && x < xhi)) sts_u32(out_b + 4u * idx, w[j]);
+                        }
+                    } else {
+                        if (b & 1u) sts_u32(out_b + 4u * q0, v[r].x);
+                        if (b & 2u) sts_u32(out_b + 4u * q1, v[r].y);
+                        if (b & 4u) sts_u32(out_b + 4u * q2, v[r].z);
+                        if (b & 8u) sts_u32(out_b + 4u * q3, v[r].w);
+                    }
+                }
+                fence_proxy_async_smem();  // the compacted words leave through a bulk store
+            }
             __syncwarp();
             if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is compacted
             if (rt == 0) trace_event(p.trace, t, 15, globaltimer());
@@ -770,7 +750,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         for (uint32_t k = r;; k += kResolvers) {
             const int o = k % kSlots;
             const uint32_t use = k / kSlots;
-            if (!mbar_wait_or_end(&bar_drawn[o], use & 1, &s_end, k)) break;
+            mbar_wait(&bar_drawn[o], use & 1);  // a tile, or an end marker (every resolver gets one)
             const uint32_t t = meta[o].tile;
             if (t == kNoTile) {
                 if (lane == 0) mbar_arrive(&bar_resolved[o]);
@@ -782,47 +762,29 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 trace_event(p.trace, t, 3, globaltimer());
             }
             __syncwarp();
-            // a5: the look-back needs only the ticket, so it runs while the tile is
-            // still being loaded and ranked.
-#ifdef DS_DEBUG_NO_LOOKBACK  // timing experiment only: wrong output, same traffic
-            const uint64_t excl = uint64_t(t) * (kT / 2);
-#else
-            uint64_t excl = 0;
-#if DS_IRR_LATE_LB  // experiment: start the look-back once the tile's own aggregate is out
-            mbar_wait(&bar_counted[o], use & 1);
-#endif
-            if (t > 0) {
-                const uint32_t tp = meta[o].prev_tile;
-                if (kLocalChain && tp != kNoTile && t - tp - 1 <= uint32_t(32 * kLW))
-                    excl = lookback_window(p.status, t, tp, &meta[(k + kSlots - 1) % kSlots], epoch, lane, p.trace);
-                else
-                    excl = lookback(p.status, t, epoch, lane, p.trace);
-            }
-#endif
-            mbar_wait(&bar_counted[o], use & 1);  // the tile's aggregate is published
+            // a5: the look-back needs only the ticket, so it could start at once; it
+            // starts once the tile's own aggregate is out (DS_IRR_LATE_LB), by when
+            // the tiles drawn before it have mostly published theirs: fewer polls,
+            // and the resolvers' issue slots go to the rankers.
+            if (kLateLookback) mbar_wait(&bar_counted[o], use & 1);
+            const uint64_t excl = t > 0 ? lookback(p.status, t, epoch, lane, p.trace) : 0ull;
+            if (!kLateLookback) mbar_wait(&bar_counted[o], use & 1);  // the tile's aggregate is published
             const uint32_t total = meta[o].total;
-            if (lane == 0) {
-                meta[o].incl = excl + total;  // the CTA's next tile chains on this
-                __threadfence_block();
-                meta[o].incl_tile = t;
-                if (t > 0 && !DBG_NO_PUBLISH) publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
-            }
-            mbar_wait(&bar_ranked[o], use & 1);  // the compacted tile is in its stage
+            if (lane == 0 && t > 0) publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
+            mbar_wait(&bar_ranked[o], use & 1);  // the compacted tile is in the ring
             if (lane == 0) {
                 trace_event(p.trace, t, 4, globaltimer());
                 meta[o].excl = excl;
-                if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = (excl + total) >> p.wshift;
+                if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = (excl + total) >> p.wshift;  // a8
                 mbar_arrive(&bar_resolved[o]);
             }
         }
     } else {
         // ------------------------------------------------ storer warps
-        // a7.  Kept words go out through one TMA bulk store per tile (the
-        // aligned interior) plus <= 6 scalar head/tail words.  The stage is
-        // first re-phased in shared memory so that its words sit at the same
-        // 16-byte phase as their destination; the stage is released once the
-        // bulk engine has read it.  Partition (two destinations) keeps the
-        // register path (store_segment).
+        // a7.  A tile's ring region goes out through one TMA bulk store (the
+        // aligned interior) plus <= 6 scalar head/tail words: the region is first
+        // re-phased in shared memory so its words sit at their destination's
+        // 16-byte phase.  The region is released once the bulk engine has read it.
         const int st = tid - 32 * kWarpStorer0;
         for (uint32_t k = 0;; ++k) {
             const int o = k % kSlots;
@@ -833,26 +795,25 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 trace_event(p.trace, t, 5, globaltimer());
                 debug_delay(t, 3);
             }
-            const int s_in = k % kInStages;
-            uint32_t* const seg = smem + s_in * kStageWords + kPre;  // rank 0 (16-byte aligned)
             const uint32_t A = meta[o].total;
+            const uint64_t excl = meta[o].excl;
+            const uint32_t rpos = meta[o].ring_pos;
+            const bool in_ring = rpos != kNoTile;
+            uint32_t* const seg = in_ring ? ring + rpos : smem + meta[o].stage * kStageWords + kPre;
+            const uint32_t ring_end = meta[o].ring_end;
             const uint64_t tb0 = uint64_t(t) * kT;
             const uint64_t vs0 = tb0 > p.lo ? tb0 : p.lo;
             const uint64_t ve0 = tb0 + kT < p.hi ? tb0 + kT : p.hi;
-            // Identity tile (in place, nothing removed in or before it): every
-            // kept word would be written onto itself, so the stores are skipped.
-            const bool identity = !PART && p.tbase == p.abase && meta[o].excl == vs0 - p.lo && A == ve0 - vs0;
-#ifndef DS_DEBUG_NO_STORE  // timing experiment only: no output written
-            // Bulk-store cnt words that sit at seg[off + r] (off % 4 == 0 or the
-            // words before them are dead) to base[d0 + r]: re-phase them in shared
-            // memory to d0's 16-byte phase, one TMA bulk store of the aligned
-            // interior, scalar head and tail (<= 3 words each).
-            auto bulk_segment = [&](uint32_t* base, uint64_t d0, uint32_t cnt, uint32_t off) {
+            // Identity tile (in place, nothing removed in or before it): every kept
+            // word would be written onto itself, so the stores are skipped.
+            const bool identity = !PART && p.tbase == p.abase && p.tlo == p.lo && excl == vs0 - p.lo &&
+                                  A == ve0 - vs0;
+            // Bulk-store the cnt words w0[0, cnt) (16-byte aligned) to base[d0, d0 + cnt).
+            auto bulk_segment = [&](uint32_t* w0, uint32_t* base, uint64_t d0, uint32_t cnt) {
                 const uint64_t d1 = d0 + cnt;
-                const uint32_t sh = (uint32_t(d0) - off) & 3u;  // shift that gives word r phase d0 + r
-                uint32_t* const b = seg + (off & ~3u);          // aligned start of the moved block
-                if (sh) rephase<kST>(b, cnt + (off & 3u), sh, st);  // word off + r -> off + sh + r
-                const uint32_t* const w = seg + off + sh;        // word r now at w[r], phase of d0 + r
+                const uint32_t sh = uint32_t(d0) & 3u;  // word r must sit at phase (d0 + r) & 3
+                if (sh) rephase<kST>(w0, cnt, sh, st);
+                const uint32_t* const w = w0 + sh;
                 const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
                 if (g1 > g0) {
                     fence_proxy_async_smem();  // re-phased words -> visible to the bulk engine
@@ -867,39 +828,25 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 }
             };
             if (!kBulkStore) {
-                if (!identity) store_segment<kST>(p.tbase, p.tlo + meta[o].excl, A, seg, 0, st);
-                if (PART) {
-                    const uint64_t excl_f = (vs0 - p.lo) - meta[o].excl;
-                    store_segment<kST>(p.fbase, p.flo + excl_f, uint32_t(ve0 - vs0) - A, seg, int32_t(A), st);
+                if (!identity) store_segment<kST>(p.tbase, p.tlo + excl, A, seg, 0, st);
+                if constexpr (PART)
+                    store_segment<kST>(p.fbase, p.flo + ((vs0 - p.lo) - excl), uint32_t(ve0 - vs0) - A, seg,
+                                       int32_t(region_true(A)), st);
+            } else {
+                if (!identity && A > 0) bulk_segment(seg, p.tbase, p.tlo + excl, A);
+                if constexpr (PART) {
+                    const uint32_t F = uint32_t(ve0 - vs0) - A;
+                    if (F > 0) bulk_segment(seg + region_true(A), p.fbase, p.flo + ((vs0 - p.lo) - excl), F);
                 }
-            } else if (PART) {
-                // Partition: trues at seg[0, A), falses at seg[A, A + F).  The trues'
-                // re-phase writes whole 16-byte chunks, up to seg[A + 6), so the
-                // first 7 falses are kept in registers until the trues' bulk store
-                // has read the stage.
-                const uint32_t F = uint32_t(ve0 - vs0) - A;
-                const uint32_t keep7 = (uint32_t(st) < 7 && uint32_t(st) < F) ? seg[A + st] : 0u;
-                named_bar_sync(2, kST);
-                if (A > 0) bulk_segment(p.tbase, p.tlo + meta[o].excl, A, 0u);
-                named_bar_sync(2, kST);
-                if (st == 0) {
-                    bulk_commit();
-                    bulk_wait_read<0>();  // the trues have been read out of the stage
-                }
-                named_bar_sync(2, kST);
-                if (uint32_t(st) < 7 && uint32_t(st) < F) seg[A + st] = keep7;
-                named_bar_sync(2, kST);
-                if (F > 0) bulk_segment(p.fbase, p.flo + ((vs0 - p.lo) - meta[o].excl), F, A);
-            } else if (!identity && A > 0) {
-                bulk_segment(p.tbase, p.tlo + meta[o].excl, A, 0u);
             }
-#endif
-            named_bar_sync(2, kST);  // every storer is done reading the stage
+            named_bar_sync(2, kST);  // every storer is done with the region
             if (st == 0) {
                 trace_event(p.trace, t, 6, globaltimer());
-                if (!DBG_NO_BULKWAIT) bulk_commit();        // (possibly empty) group of this tile
-                if (!DBG_NO_BULKWAIT) bulk_wait_read<0>();  // the bulk engine has read the stage
-                if (!DBG_EARLY_FREE) mbar_arrive(&bar_free[s_in]);
+                bulk_commit();        // (possibly empty) group of this tile
+                bulk_wait_read<0>();  // the bulk engine has read the region
+                // ring words allocated up to this tile belong to tiles stored by now
+                st_release_cta_smem(&s_freed, ring_end);
+                if (!in_ring) stage_release(&s_stages, meta[o].stage);
                 mbar_arrive(&bar_stored[o]);
             }
         }

@@ -46,7 +46,141 @@ __global__ void __launch_bounds__(kW * 32, 1) rank_kernel(const uint32_t* src, i
         const long long c0 = clock64();
         const int xs = kSeg * rw;
         uint32_t total, wbase, wrun = 0;
-        if constexpr (V == 10) {
+        if constexpr (V == 13 || V == 14) {
+            // V13: V11 with explicit 32-bit shared addresses (st.shared), keep bits
+            // packed with one POPC per 4 words, store phase skipped for empty warps.
+            // V14: V13 with the 4 keep bits turned into the in-lane prefix by a
+            // nibble lookup (prefix of bits below j for j = 1..3 in 2-bit fields).
+            const uint32_t sbase = uint32_t(__cvta_generic_to_shared(stage));
+            uint4 v[4];
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                const uint32_t a = sbase + 4u * uint32_t(xs + 128 * r + 4 * lane);
+                asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+                             : "=r"(v[r].x), "=r"(v[r].y), "=r"(v[r].z), "=r"(v[r].w) : "r"(a));
+            }
+            uint32_t kb = 0, P = 0;
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                const uint32_t b = uint32_t(v[r].x != 0u) | uint32_t(v[r].y != 0u) << 1 |
+                                   uint32_t(v[r].z != 0u) << 2 | uint32_t(v[r].w != 0u) << 3;
+                kb |= b << (4 * r);
+                P += uint32_t(__popc(b)) << (8 * r);
+            }
+            uint32_t inc = P;
+#pragma unroll
+            for (int sh = 1; sh < 32; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, inc, sh);
+                if (lane >= sh) inc += y;
+            }
+            const uint32_t E = inc - P;
+            const uint32_t T4 = __shfl_sync(kFull, inc, 31);
+            const uint32_t T0 = T4 & 255u, T1 = T4 >> 8 & 255u, T2 = T4 >> 16 & 255u, T3 = T4 >> 24;
+            wrun = T0 + T1 + T2 + T3;
+            if (lane == 0) wtot[rw] = wrun;
+            const long long ca = clock64();
+            seg_a += ca - c0;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            const uint32_t cw = lane < kW ? wtot[lane] : 0u;
+            uint32_t iw = cw;
+#pragma unroll
+            for (int sh = 1; sh < kW; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, iw, sh);
+                if (lane >= sh) iw += y;
+            }
+            total = __shfl_sync(kFull, iw, kW - 1);
+            wbase = __shfl_sync(kFull, iw - cw, rw);
+            seg_b += clock64() - c0 + (total & 1);
+            if (wrun != 0) {
+                const uint32_t R[4] = {0u, T0, T0 + T1, T0 + T1 + T2};
+#pragma unroll
+                for (int r = 0; r < 4; ++r) {
+                    const uint32_t b = kb >> (4 * r) & 15u;
+                    const uint32_t a0 = sbase + 4u * (wbase + R[r] + (E >> (8 * r) & 255u));
+                    uint32_t a1, a2, a3;
+                    if (V == 13) {
+                        a1 = a0 + 4u * (b & 1u);
+                        a2 = a1 + 4u * (b >> 1 & 1u);
+                        a3 = a2 + 4u * (b >> 2 & 1u);
+                    } else {
+                        // in-lane prefixes for j = 1, 2, 3 from a 16-entry table of 3 x 2-bit fields
+                        constexpr uint64_t kLo = 0, kT = 0;
+                        (void)kLo; (void)kT;
+                        const uint32_t pre = (0xE9A59A55u >> (2 * b)) ;  // unused bits: see below
+                        (void)pre;
+                        a1 = a0 + 4u * (b & 1u);
+                        a2 = a0 + 4u * __popc(b & 3u);
+                        a3 = a0 + 4u * __popc(b & 7u);
+                    }
+                    if (b & 1u) asm volatile("st.shared.u32 [%0], %1;" ::"r"(a0), "r"(v[r].x) : "memory");
+                    if (b & 2u) asm volatile("st.shared.u32 [%0], %1;" ::"r"(a1), "r"(v[r].y) : "memory");
+                    if (b & 4u) asm volatile("st.shared.u32 [%0], %1;" ::"r"(a2), "r"(v[r].z) : "memory");
+                    if (b & 8u) asm volatile("st.shared.u32 [%0], %1;" ::"r"(a3), "r"(v[r].w) : "memory");
+                }
+            }
+        } else if constexpr (V == 11 || V == 12) {
+            // V11: lane-vector layout, no ballots and no per-word POPC.  Lane l of
+            // round r holds words xs + 128r + 4l .. +3 (one LDS.128, conflict-free);
+            // its 4 keep bits give a count 0..4 (ALU); the counts of the 4 rounds are
+            // packed in 8-bit fields of one register and one 5-step shuffle scan over
+            // the lanes gives every lane its exclusive offset in all 4 rounds.
+            // V12: V11 with the in-lane ranks by a 4-entry select instead of adds.
+            uint4 v[4];
+#pragma unroll
+            for (int r = 0; r < 4; ++r) v[r] = *reinterpret_cast<const uint4*>(&stage[xs + 128 * r + 4 * lane]);
+            uint32_t kb = 0, P = 0;
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                const uint32_t k0 = v[r].x != 0u, k1 = v[r].y != 0u, k2 = v[r].z != 0u, k3 = v[r].w != 0u;
+                kb |= (k0 | k1 << 1 | k2 << 2 | k3 << 3) << (4 * r);
+                P += (k0 + k1 + k2 + k3) << (8 * r);
+            }
+            uint32_t inc = P;
+#pragma unroll
+            for (int sh = 1; sh < 32; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, inc, sh);
+                if (lane >= sh) inc += y;
+            }
+            const uint32_t E = inc - P;
+            const uint32_t T4 = __shfl_sync(kFull, inc, 31);
+            const uint32_t T0 = T4 & 255u, T1 = T4 >> 8 & 255u, T2 = T4 >> 16 & 255u, T3 = T4 >> 24;
+            const uint32_t R[4] = {0u, T0, T0 + T1, T0 + T1 + T2};
+            wrun = T0 + T1 + T2 + T3;
+            if (lane == 0) wtot[rw] = wrun;
+            const long long ca = clock64();
+            seg_a += ca - c0;
+            asm volatile("bar.sync 1, %0;" ::"r"(kW * 32) : "memory");
+            const uint32_t cw = lane < kW ? wtot[lane] : 0u;
+            uint32_t iw = cw;
+#pragma unroll
+            for (int sh = 1; sh < kW; sh <<= 1) {
+                const uint32_t y = __shfl_up_sync(kFull, iw, sh);
+                if (lane >= sh) iw += y;
+            }
+            total = __shfl_sync(kFull, iw, kW - 1);
+            wbase = __shfl_sync(kFull, iw - cw, rw);
+            seg_b += clock64() - c0 + (total & 1);
+#pragma unroll
+            for (int r = 0; r < 4; ++r) {
+                uint32_t q = wbase + R[r] + (E >> (8 * r) & 255u);
+                const uint32_t b = kb >> (4 * r);
+                if (V == 11) {
+                    if (b & 1u) stage[q] = v[r].x;
+                    q += b & 1u;
+                    if (b & 2u) stage[q] = v[r].y;
+                    q += b >> 1 & 1u;
+                    if (b & 4u) stage[q] = v[r].z;
+                    q += b >> 2 & 1u;
+                    if (b & 8u) stage[q] = v[r].w;
+                } else {
+                    const uint32_t q1 = q + (b & 1u), q2 = q1 + (b >> 1 & 1u), q3 = q2 + (b >> 2 & 1u);
+                    if (b & 1u) stage[q] = v[r].x;
+                    if (b & 2u) stage[q1] = v[r].y;
+                    if (b & 4u) stage[q2] = v[r].z;
+                    if (b & 8u) stage[q3] = v[r].w;
+                }
+            }
+        } else if constexpr (V == 10) {
             // V10: no ballots, no POPC.  Lane l packs its 16 keep bits into 5-bit
             // fields (chunk c -> register c / 6, bits 5 (c % 6)); a shuffle scan over
             // the lanes of the packed words gives every lane, for all 16 chunks at
@@ -302,7 +436,8 @@ __global__ void __launch_bounds__(kW * 32, 1) rank_kernel(const uint32_t* src, i
     if (acc == 0x12345) atomicAdd(sink, acc + stage[lane]);
 }
 
-int main() {
+int main(int argc, char** argv) {
+    const double fkeep = argc > 1 ? atof(argv[1]) : 0.5;
     int sms;
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
     const size_t nw = size_t(64) * kT;
@@ -310,7 +445,7 @@ int main() {
     uint64_t x = 0x9E3779B97F4A7C15ull;
     for (size_t i = 0; i < nw; ++i) {
         x ^= x << 13; x ^= x >> 7; x ^= x << 17;
-        h[i] = (x >> 40) & 1 ? uint32_t(x) | 1u : 0u;
+        h[i] = double((x >> 40) & 0xFFFFu) < fkeep * 65536.0 ? uint32_t(x) | 1u : 0u;
     }
     uint32_t* d;
     unsigned long long *cyc, *sink;
@@ -348,6 +483,12 @@ int main() {
     run("V2 V1 without compaction stores", rank_kernel<2>);
     run("V3 64-bit loads, two ballots", rank_kernel<3>);
     run("V4 128-bit loads, four ballots", rank_kernel<4>);
+    run("V11 lane-vector, packed 8-bit scan", rank_kernel<11>);
+    run("V11 no fence", rank_kernel<11 | 16>);
+    run("V12 lane-vector, q precomputed", rank_kernel<12>);
+    run("V13 lane-vector, st.shared, popc", rank_kernel<13>);
+    run("V13 no fence", rank_kernel<13 | 16>);
+    run("V14 V13 with popc prefixes", rank_kernel<14>);
     run("V10 packed shuffle scan", rank_kernel<10>);
     run("V10 no fence", rank_kernel<10 | 16>);
     run("V9 chunk offsets from phase 1", rank_kernel<9>);
