@@ -114,7 +114,7 @@ struct OpUnique64 {
 };
 
 // ---- CTA shape ----------------------------------------------------------
-// warps: 16 rankers (2 groups of 8) | 4 resolvers | 4 storers | 1 producer
+// warps: 16 rankers (2 groups of 8) | 4 resolvers | 3 storers | 1 producer
 #ifndef DS_IRR_IN_STAGES
 #define DS_IRR_IN_STAGES 4
 #endif
@@ -125,7 +125,7 @@ struct OpUnique64 {
 #define DS_IRR_RESOLVERS 4
 #endif
 #ifndef DS_IRR_STORE_WARPS
-#define DS_IRR_STORE_WARPS 4
+#define DS_IRR_STORE_WARPS 3
 #endif
 #ifndef DS_IRR_BULK_STORE
 #define DS_IRR_BULK_STORE 1
@@ -565,6 +565,9 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             uint32_t kb = 0, P[kPacks];
 #pragma unroll
             for (int i = 0; i < kPacks; ++i) P[i] = 0;
+            // unique: rot[r] = lane l-1's last word of round r; lane 0 receives lane 31's,
+            // which is lane 0's predecessor in round r+1 (one shuffle per round)
+            uint32_t rot_z = 0, rot_w = 0;
 #pragma unroll
             for (int r = 0; r < kRounds; ++r) {
                 const uint32_t x0 = uint32_t(xs + 128 * r + 4 * lane);
@@ -574,16 +577,17 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                     if constexpr (Op::kUnique) {
                         // element before (x, y): lane l-1's (z, w), lane 31 of the previous
                         // round, or the two staged words before the segment
-                        pz = __shfl_up_sync(kFull, v[r].z, 1);
-                        pw = __shfl_up_sync(kFull, v[r].w, 1);
-                        if (r > 0) {
-                            const uint32_t lz = __shfl_sync(kFull, v[r > 0 ? r - 1 : 0].z, 31);
-                            const uint32_t lw = __shfl_sync(kFull, v[r > 0 ? r - 1 : 0].w, 31);
-                            if (lane == 0) pz = lz, pw = lw;
-                        } else if (lane == 0) {
+                        const uint32_t tz = __shfl_sync(kFull, v[r].z, (lane + 31) & 31);
+                        const uint32_t tw = __shfl_sync(kFull, v[r].w, (lane + 31) & 31);
+                        if (lane != 0) {
+                            pz = tz, pw = tw;
+                        } else if (r > 0) {
+                            pz = rot_z, pw = rot_w;
+                        } else {
                             pz = lds_u32(st_b + 4u * uint32_t(xs - 2));
                             pw = lds_u32(st_b + 4u * uint32_t(xs - 1));
                         }
+                        rot_z = tz, rot_w = tw;
                     }
                     b = keep_bits4_wide<Op>(v[r], pz, pw, uint64_t(p.value_hi) << 32 | p.value);
                     if (Op::kUnique && guarded && t == 0) {  // the array's first element is kept
@@ -595,13 +599,9 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                     if constexpr (Op::kUnique) {
                         // word before x0: lane l-1's last word, lane 31 of the previous
                         // round, or the staged word before the segment (P:280 for xs = 0)
-                        pw = __shfl_up_sync(kFull, v[r].w, 1);
-                        if (r > 0) {
-                            const uint32_t lw = __shfl_sync(kFull, v[r > 0 ? r - 1 : 0].w, 31);
-                            if (lane == 0) pw = lw;
-                        } else if (lane == 0) {
-                            pw = lds_u32(st_b + 4u * uint32_t(xs - 1));
-                        }
+                        const uint32_t tw = __shfl_sync(kFull, v[r].w, (lane + 31) & 31);
+                        pw = lane != 0 ? tw : r > 0 ? rot_w : lds_u32(st_b + 4u * uint32_t(xs - 1));
+                        rot_w = tw;
                     }
                     b = keep_bits4<Op>(v[r], pw, p.value);
                     if (Op::kUnique && guarded && t == 0 && x0 <= xlo && xlo < x0 + 4) {

@@ -8,7 +8,7 @@ Prints, over all tiles, percentiles of the stage latencies (us):
   cwait    cstart - incl           (waiting for the CTA's consumers)
   consume  cend - cstart           (rank, scatter, stores issued)
 and the overall tile rate.
-    python tools/trace_pipeline.py [n_log2] [f]
+    [DS_OP=unique] python tools/trace_pipeline.py [n_log2] [f]
 """
 import os
 import sys
@@ -27,7 +27,11 @@ def main():
     lg = int(sys.argv[1]) if len(sys.argv) > 1 else 28
     f = float(sys.argv[2]) if len(sys.argv) > 2 else 0.5
     n = 1 << lg
-    src = dsgen.compact_input(n, f, 7, device="cuda")
+    op = os.environ.get("DS_OP", "compact")
+    if op == "unique":
+        src = dsgen.unique_runs_input(n, f, 5, device="cuda")
+    else:
+        src = dsgen.compact_input(n, f, 7, device="cuda")
     work = torch.empty_like(src)
     ntiles = (n + T - 1) // T
     tr = torch.zeros(ntiles * 16, dtype=torch.int64, device="cuda")
@@ -36,7 +40,10 @@ def main():
         work.copy_(src)
         torch.cuda.synchronize()
         libds.ds_debug_set_trace(tr if rep == 2 else None, ntiles if rep == 2 else 0)
-        libds.ds_compact_ex(work, n, 0, d_n, None)
+        if op == "unique":
+            libds.ds_unique_ex(work, n, None, 0, d_n, None)
+        else:
+            libds.ds_compact_ex(work, n, 0, d_n, None)
         torch.cuda.synchronize()
     libds.ds_debug_set_trace(None, 0)
     t = tr.cpu().numpy().reshape(ntiles, 16).astype(np.int64)
