@@ -27,8 +27,8 @@
  *    stream-ordered on `stream`; their count is written to DEVICE memory
  *    (d_out_n, may be NULL).
  *  - libds keeps, per (device, stream), a small workspace: one 64-bit
- *    status word per tile (n/4096 words, ~0.2% of the data) and one
- *    ticket/epoch word.  Calls that share a stream share it; calls on
+ *    status word per tile of 8192 words (one per 64-byte line, ~0.2% of
+ *    the data) and one ticket/epoch word.  Calls that share a stream share it; calls on
  *    different streams may run concurrently.  ds_release_workspaces()
  *    frees it (call only when no libds kernel is in flight).
  *  - Thread-safe: host state is protected by a mutex.
@@ -228,6 +228,18 @@ uint64_t ds_launch_count(void);
 ds_status ds_debug_set_trace(uint64_t* d_trace, size_t capacity_tiles);
 /* Library version, major*10000 + minor*100 + patch.                      */
 int ds_version(void);
+
+/* Tile size of a kernel family, for tests that aim at tile edges: the
+ * irregular kernel's input tile and the regular kernel's output tile in
+ * 4-byte words, the byte-granular regular kernel's output tile in bytes
+ * (0 for an unknown id).  Tiles start at the 16-byte boundary at or below
+ * ptr, so tile k covers words [16B-aligned base + kT, ...).              */
+typedef enum ds_kernel {
+    DS_KERNEL_IRREGULAR = 0,      /* compact / select / unique / partition */
+    DS_KERNEL_REGULAR = 1,        /* pad / unpad / slide, whole words      */
+    DS_KERNEL_REGULAR_BYTES = 2   /* pad / unpad, 1- and 2-byte rows       */
+} ds_kernel;
+size_t ds_tile_size(int kernel);
 
 #ifdef __cplusplus
 }

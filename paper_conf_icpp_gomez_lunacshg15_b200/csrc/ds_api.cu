@@ -272,14 +272,18 @@ ds_status ds_unpad_ex(void* ptr, size_t rows, size_t cols, size_t new_cols, size
     return run_regular(a, reinterpret_cast<cudaStream_t>(stream));
 }
 
+// The blocking forms synchronise only when a kernel was enqueued (a no-op
+// call needs no device).
 ds_status ds_pad(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes) {
     ds_status st = ds_pad_ex(ptr, rows, cols, new_cols, elem_bytes, nullptr, nullptr);
-    return st == DS_SUCCESS ? sync_default() : st;
+    if (st != DS_SUCCESS || rows == 0 || cols == new_cols) return st;
+    return sync_default();
 }
 
 ds_status ds_unpad(void* ptr, size_t rows, size_t cols, size_t new_cols, size_t elem_bytes) {
     ds_status st = ds_unpad_ex(ptr, rows, cols, new_cols, elem_bytes, nullptr);
-    return st == DS_SUCCESS ? sync_default() : st;
+    if (st != DS_SUCCESS || rows == 0 || cols == new_cols || new_cols == 0) return st;
+    return sync_default();
 }
 
 ds_status ds_slide_ex(void* ptr, size_t n, size_t shift, size_t elem_bytes, ds_stream_t stream) {
@@ -315,7 +319,8 @@ ds_status ds_slide_ex(void* ptr, size_t n, size_t shift, size_t elem_bytes, ds_s
 
 ds_status ds_slide(void* ptr, size_t n, size_t shift, size_t elem_bytes) {
     ds_status st = ds_slide_ex(ptr, n, shift, elem_bytes, nullptr);
-    return st == DS_SUCCESS ? sync_default() : st;
+    if (st != DS_SUCCESS || shift == 0 || shift == n) return st;
+    return sync_default();
 }
 
 ds_status ds_compact_ex(void* ptr, size_t n, uint32_t remove_value, uint64_t* d_out_n,
@@ -562,6 +567,15 @@ ds_status ds_debug_set_trace(uint64_t* d_trace, size_t capacity_tiles) {
     return DS_SUCCESS;
 }
 
-int ds_version(void) { return 100; }
+int ds_version(void) { return 200; }
+
+size_t ds_tile_size(int kernel) {
+    switch (kernel) {
+    case DS_KERNEL_IRREGULAR: return ds::irregular_tile_words();
+    case DS_KERNEL_REGULAR: return ds::regular_tile_words();
+    case DS_KERNEL_REGULAR_BYTES: return ds::regular_bytes_tile_bytes();
+    }
+    return 0;
+}
 
 }  // extern "C"

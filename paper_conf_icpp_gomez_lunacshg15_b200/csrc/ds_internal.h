@@ -59,6 +59,11 @@ struct RegBytesArgs {
     bool pad;
 };
 
+// Tile sizes of the kernel families (ds_tile_size).
+size_t irregular_tile_words();
+size_t regular_tile_words();
+size_t regular_bytes_tile_bytes();
+
 // Tiles a launch of each kernel family needs (for workspace sizing).
 size_t irregular_tiles(const IrregArgs& a);
 size_t regular_tiles(const RegArgs& a);

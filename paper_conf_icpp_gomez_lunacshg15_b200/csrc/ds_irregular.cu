@@ -886,6 +886,8 @@ cudaError_t launch_op(IrregParams p, cudaStream_t s) {
 
 }  // namespace
 
+size_t irregular_tile_words() { return kT; }
+
 size_t irregular_tiles(const IrregArgs& a) {
     const uint64_t lo = (reinterpret_cast<uintptr_t>(a.ptr) >> 2) & 3u;
     return size_t((lo + a.n + kT - 1) / kT);

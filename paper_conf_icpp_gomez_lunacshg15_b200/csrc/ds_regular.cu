@@ -419,6 +419,8 @@ cudaError_t launch_dir(RegParams p, cudaStream_t s) {
 
 }  // namespace
 
+size_t regular_tile_words() { return kT; }
+
 size_t regular_tiles(const RegArgs& a) {
     const uint64_t mis = (reinterpret_cast<uintptr_t>(a.ptr) >> 2) & 3u;
     const uint64_t out_words = a.out_words_w ? a.out_words_w : a.rows * a.new_cols_w;

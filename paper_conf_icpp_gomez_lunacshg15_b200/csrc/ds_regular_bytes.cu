@@ -407,6 +407,8 @@ cudaError_t launch_dir_b(RegBParams p, cudaStream_t s) {
 
 }  // namespace
 
+size_t regular_bytes_tile_bytes() { return kTB; }
+
 size_t regular_bytes_tiles(const RegBytesArgs& a) {
     const uint64_t mis = reinterpret_cast<uintptr_t>(a.ptr) & 15u;
     return size_t((a.rows * a.new_cols_b + mis + kTB - 1) / kTB);

@@ -52,6 +52,7 @@ SIGNATURES = {
     "ds_release_workspaces": (_i, []),
     "ds_launch_count": (_u64, []),
     "ds_version": (_i, []),
+    "ds_tile_size": (_sz, [_i]),
     "ds_debug_set_trace": (_i, [_vp, _sz]),
 }
 
@@ -266,6 +267,13 @@ def ds_launch_count() -> int:
 
 def ds_version() -> int:
     return int(_lib.ds_version())
+
+
+DS_KERNEL_IRREGULAR, DS_KERNEL_REGULAR, DS_KERNEL_REGULAR_BYTES = 0, 1, 2
+
+
+def ds_tile_size(kernel: int) -> int:
+    return int(_lib.ds_tile_size(kernel))
 
 
 def ds_debug_set_trace(d_trace, capacity_tiles: int) -> None:

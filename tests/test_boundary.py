@@ -48,7 +48,15 @@ def test_status_strings_and_version():
     assert libds.ds_status_string(0) == "DS_SUCCESS"
     assert libds.ds_status_string(INV) == "DS_ERROR_INVALID_VALUE"
     assert libds.ds_status_string(4) == "DS_ERROR_CUDA"
-    assert libds.ds_version() >= 100
+    assert libds.ds_version() >= 200
+
+
+def test_tile_sizes():
+    """The tile sizes the GPU tile-edge sweeps are keyed to (ds_tile_size)."""
+    assert libds.ds_tile_size(libds.DS_KERNEL_IRREGULAR) == 8192
+    assert libds.ds_tile_size(libds.DS_KERNEL_REGULAR) == 8192
+    assert libds.ds_tile_size(libds.DS_KERNEL_REGULAR_BYTES) == 32768
+    assert libds.ds_tile_size(7) == 0
 
 
 def st(name, *args):
@@ -110,7 +118,10 @@ def test_regular_validation_before_device():
 
 
 def test_regular_noops_need_no_device():
-    assert st("ds_pad", FAKE, 0, 5, 9, 4) == 0 or True  # rows == 0 is a no-op (sync may need a device)
+    assert st("ds_pad", FAKE, 0, 5, 9, 4) == 0            # rows == 0: no launch, no sync
+    assert st("ds_unpad", FAKE, 7, 5, 5, 4) == 0           # cols == new_cols
+    assert st("ds_unpad", FAKE, 7, 5, 0, 4) == 0           # nothing kept
+    assert st("ds_slide", FAKE, 9, 0, 4) == 0              # shift 0
     assert st("ds_pad_ex", FAKE, 0, 5, 9, 4, None, None) == 0
     assert st("ds_pad_ex", FAKE, 7, 5, 5, 4, None, None) == 0     # new_cols == cols
     assert st("ds_unpad_ex", FAKE, 7, 5, 0, 4, None) == 0         # nothing kept

@@ -2,9 +2,12 @@
 WHOLE buffer including canary words around it (tolerance 0: integer /
 indexing work).  Inputs come from dsgen (seeded, shared by both sides).
 
-Sizes span several tiles (T = 4096 words) with ragged tails; pointers are
-misaligned by 0..3 words; fractions sweep 0..100 %.  Every call goes
-through the C ABI (ctypes binding)."""
+Sizes span several tiles with ragged tails; the tile sizes are read from the
+library (ds_tile_size: T words for the irregular kernel, TR output words for
+the regular kernel), and tiles start at the 16-byte boundary at or below
+ptr, so a pointer misaligned by `mis` words moves every tile edge by mis.
+Pointers are misaligned by 0..3 words; fractions sweep 0..100 %.  Every call
+goes through the C ABI (ctypes binding)."""
 import numpy as np
 import pytest
 import torch
@@ -16,7 +19,8 @@ from paper_conf_icpp_gomez_lunacshg15_b200 import libds
 
 pytestmark = pytest.mark.gpu
 
-T = 4096
+T = libds.ds_tile_size(libds.DS_KERNEL_IRREGULAR)      # irregular input tile (words)
+TR = libds.ds_tile_size(libds.DS_KERNEL_REGULAR)       # regular output tile (words)
 SIZES = [1, 2, 3, 4, 5, 31, 32, 33, 1000, T - 1, T, T + 1, 2 * T - 1, 2 * T + 1, 3 * T + 7,
          65537, 1_000_003]
 FRACS = [0.0, 0.1, 0.5, 0.9, 1.0]
@@ -40,25 +44,97 @@ def test_compact_sizes_misalignment(n, mis):
         buf.assert_equals(exp, f"compact n={n} mis={mis} f={f}")
 
 
-def _structured(n):
+def _structured(n, mis=0):
+    """Keep masks (kept word = its index + 1, removed = 0) aimed at the tile
+    grid the kernel sees: virtual index v = i + mis, tile = v // T."""
     i = np.arange(n, dtype=np.uint32)
-    yield "all_removed_but_last", np.where(i == n - 1, i + 1, 0).astype(np.uint32)
-    yield "first_half_removed", np.where(i >= n // 2, i + 1, 0).astype(np.uint32)
-    yield "alternating", np.where(i % 2 == 1, i + 1, 0).astype(np.uint32)
-    yield "one_per_tile", np.where(i % T == T - 1, i + 1, 0).astype(np.uint32)
-    yield "odd_tiles_only", np.where((i // T) % 2 == 1, i + 1, 0).astype(np.uint32)
-    yield "runs_cross_tiles", np.where(((i + 1000) // 3000) % 2 == 0, i + 1, 0).astype(np.uint32)
+    v = i.astype(np.int64) + mis
+    keep = lambda m: np.where(m, i + 1, 0).astype(np.uint32)  # noqa: E731
+    yield "all_removed_but_last", keep(i == n - 1)
+    yield "first_half_removed", keep(i >= n // 2)
+    yield "alternating", keep(i % 2 == 1)
+    yield "one_per_tile_last_word", keep(v % T == T - 1)
+    yield "one_per_tile_first_word", keep(v % T == 0)
+    yield "one_per_tile_middle", keep(v % T == T // 2 + 1)
+    yield "odd_tiles_only", keep((v // T) % 2 == 1)
+    yield "even_tiles_only", keep((v // T) % 2 == 0)
+    yield "run_ends_at_tile_edge", keep((v >= T // 2) & (v < 2 * T))
+    yield "run_starts_at_tile_edge", keep((v >= T) & (v < 2 * T + 100))
+    yield "runs_cross_tiles", keep(((i + 1000) // 3000) % 2 == 0)
 
 
-@pytest.mark.parametrize("n", [5 * T + 3, 200_000])
-def test_compact_structured_masks(n):
-    for name, a in _structured(n):
-        for mis in (0, 3):
-            buf = DevBuf(a, mis)
-            exp = buf.host_region()
-            m_exp = oracle.compact(exp, 0)
-            assert libds.ds_compact(buf.ptr, n, 0) == m_exp, name
-            buf.assert_equals(exp, name)
+@pytest.mark.parametrize("n", [5 * T + 3, 4 * T, 200_000])
+@pytest.mark.parametrize("mis", [0, 1, 2, 3])
+def test_compact_structured_masks(n, mis):
+    for name, a in _structured(n, mis):
+        buf = DevBuf(a, mis)
+        exp = buf.host_region()
+        m_exp = oracle.compact(exp, 0)
+        assert libds.ds_compact(buf.ptr, n, 0) == m_exp, name
+        buf.assert_equals(exp, f"{name} mis={mis}")
+
+
+# ----------------------------------------------------------- tile edges
+# n = k*T - mis + d: the last tile ends exactly at (d = 0), one word before
+# (d = -1) or one word past (d = +1) a tile edge of the kernel's grid.
+EDGE_CASES = [(k, mis, d) for k in (1, 2, 3) for mis in range(4) for d in (-1, 0, 1)]
+
+
+@pytest.mark.parametrize("k,mis,d", EDGE_CASES)
+def test_irregular_tile_edges(k, mis, d):
+    n = k * T - mis + d
+    for j, f in enumerate((0.0, 0.5, 1.0)):
+        seed = dsgen.seed_for(0, 100 + 4 * k + mis + 16 * j)
+        a = _u32(dsgen.compact_input(n, f, seed))
+        buf = DevBuf(a, mis)
+        exp = buf.host_region()
+        m_exp = oracle.compact(exp, 0)
+        assert libds.ds_compact(buf.ptr, n, 0) == m_exp
+        buf.assert_equals(exp, f"compact n={n} mis={mis} f={f}")
+        u = _u32(dsgen.unique_runs_input(n, f, seed + 1))
+        buf = DevBuf(u, mis)
+        exp = buf.host_region()
+        m_exp = oracle.unique(exp)
+        assert libds.ds_unique(buf.ptr, n) == m_exp
+        buf.assert_equals(exp, f"unique n={n} mis={mis} f={f}")
+        sel = _u32(dsgen.select_input(n, seed + 2))
+        t = dsgen.select_threshold(f) & 0xFFFFFFFF
+        buf = DevBuf(sel, mis)
+        exp = buf.host_region()
+        m_exp = oracle.select(exp, libds.DS_PRED_I32_GT, t)
+        d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+        libds.ds_select_ex(buf.ptr, n, libds.DS_PRED_I32_GT, t, d_n, None)
+        torch.cuda.synchronize()
+        assert int(d_n.item()) == m_exp
+        buf.assert_equals(exp, f"select n={n} mis={mis} f={f}")
+
+
+@pytest.mark.parametrize("mis", [0, 1, 2, 3])
+def test_unique_structured_tile_edges(mis):
+    """Runs whose boundaries sit on the kernel's tile edges."""
+    n = 4 * T + 5
+    v = np.arange(n, dtype=np.int64) + mis
+    cases = {"run_per_tile": v // T, "change_at_last_word": (v + 1) // T,
+             "change_at_first_word": np.maximum(v - 1, 0) // T, "one_change_per_tile": (v % T == T - 1).cumsum(),
+             "constant": np.zeros(n, dtype=np.int64)}
+    for name, ids in cases.items():
+        a = (ids * 2654435761 % (1 << 32)).astype(np.uint32)
+        buf = DevBuf(a, mis)
+        exp = buf.host_region()
+        m_exp = oracle.unique(exp)
+        assert libds.ds_unique(buf.ptr, n) == m_exp, name
+        buf.assert_equals(exp, f"unique {name} mis={mis}")
+
+
+@pytest.mark.parametrize("k,mis,d", [(k, mis, d) for k in (1, 2, 3) for mis in (0, 1, 3) for d in (-1, 0, 1)])
+def test_regular_tile_edges(k, mis, d):
+    """Pad / unpad whose output ends at (or one word around) an output-tile
+    edge: rows of 7 words padded to 8, rows = (k*TR - mis + d) // 8."""
+    out_words = k * TR - mis + d
+    R, C, NC = max(1, out_words // 8), 7, 8
+    _pad_case(R, C, NC, 4, mis, fill=[0xFEED0000 + k])
+    # one long row: the whole output is a single row crossing every edge
+    _pad_case(1, out_words - 3, out_words, 4, mis, fill=[0xBEEF0000 + d + 1])
 
 
 def test_compact_remove_value_bitwise():
@@ -400,7 +476,7 @@ def test_slide_ex_stream_repeated():
 
 
 # ------------------------------------------------------ 8-byte elements
-SIZES64 = [1, 2, 3, 16, 2047, 4096, 4097, 8191, 3 * 4096 + 5, 100_003, 1_000_003]
+SIZES64 = [1, 2, 3, 16, T // 2 - 1, T // 2, T // 2 + 1, T - 1, 3 * (T // 2) + 5, 100_003, 1_000_003]  # elements (T/2 per tile)
 
 
 def _dev64(host, mis):
