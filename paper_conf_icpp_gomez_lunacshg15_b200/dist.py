@@ -26,12 +26,22 @@ and slide, so the ranks go in "waves" (wave = 1 + the largest wave of the
 ranks it sends to); each wave is one batch of NCCL send/recv over NVLink.
 
 The device steps are delegated to a ``local`` object; the default,
-``LibdsLocal``, calls the libds C ABI on CUDA tensors.  Tests substitute a
-CPU stand-in to exercise the orchestration and the collectives with gloo.
+``LibdsLocal``, calls the libds C ABI on CUDA tensors.  The two collectives
+(all-gather of 8-byte values, the rebalance's point-to-point pieces) go
+through a ``comm`` object; the default, ``DistComm``, runs them on the
+process group (NCCL over NVLink on a GPU box) on the device tensors.  Tests
+substitute a CPU stand-in for ``local`` (orchestration over gloo) and a
+CPU-staged gloo ``comm`` (the real kernels, several ranks on one GPU).
+
+Stream ordering: every call takes the stream the libds kernels run on (None
+= torch's current stream).  The collectives are issued with that stream
+current, so they start after the kernels before them on it, and the work
+after them on it (offsets kernel, slide) waits for them.
 """
 from __future__ import annotations
 
 import bisect
+import contextlib
 from dataclasses import dataclass
 
 import torch
@@ -74,6 +84,26 @@ class LibdsLocal:
 
     def slide(self, shard, n, shift, stream=None):
         self.libds.ds_slide_ex(shard if n else None, n, shift, 4, stream)
+
+
+class DistComm:
+    """Collectives on the process group, on device tensors (NCCL on a GPU box).
+    Issued with the caller's stream current (ShardedDS), so torch orders the
+    NCCL stream after it and, through req.wait(), it after the NCCL stream."""
+
+    def __init__(self, group=None):
+        self.group = group
+
+    def all_gather(self, out: torch.Tensor, inp: torch.Tensor) -> None:
+        dist.all_gather_into_tensor(out, inp, group=self.group)
+
+    def exchange(self, sends, recvs) -> None:
+        """sends / recvs: lists of (tensor, peer rank); one batched round."""
+        ops = [dist.P2POp(dist.isend, t, peer, self.group) for t, peer in sends]
+        ops += [dist.P2POp(dist.irecv, t, peer, self.group) for t, peer in recvs]
+        if ops:
+            for req in dist.batch_isend_irecv(ops):
+                req.wait()
 
 
 @dataclass(frozen=True)
@@ -142,12 +172,13 @@ class ShardResult:
 class ShardedDS:
     """One rank's view of a sharded in-place DS operation."""
 
-    def __init__(self, group=None, device=None, local=None):
+    def __init__(self, group=None, device=None, local=None, comm=None):
         self.group = group
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
         self.device = torch.device(device) if device is not None else torch.device("cuda")
         self.local = local if local is not None else LibdsLocal()
+        self.comm = comm if comm is not None else DistComm(group)
         self.d_count = self.local.alloc_u64(1, self.device)
         self.d_counts = self.local.alloc_u64(self.world, self.device)
         self.d_result = self.local.alloc_u64(2, self.device)
@@ -155,14 +186,24 @@ class ShardedDS:
         self.d_halo = self.local.alloc_u64(self.world, self.device)
         self._sizes = None  # every rank's shard capacity (rebalance), gathered once
 
-    def _allgather(self, out: torch.Tensor, inp: torch.Tensor) -> None:
-        if self.world == 1:
-            out.copy_(inp)
-        else:
-            dist.all_gather_into_tensor(out, inp, group=self.group)
+    @staticmethod
+    def _on(stream):
+        """Issue torch work (collectives, copies) on the libds stream."""
+        if isinstance(stream, torch.cuda.Stream):
+            return torch.cuda.stream(stream)
+        if stream is not None:
+            raise TypeError("ShardedDS needs a torch.cuda.Stream (or None for the current stream)")
+        return contextlib.nullcontext()
+
+    def _allgather(self, out: torch.Tensor, inp: torch.Tensor, stream=None) -> None:
+        with self._on(stream):
+            if self.world == 1:
+                out.copy_(inp)
+            else:
+                self.comm.all_gather(out, inp)
 
     def _finish(self, stream) -> ShardResult:
-        self._allgather(self.d_counts, self.d_count)
+        self._allgather(self.d_counts, self.d_count, stream)
         self.local.offsets(self.d_counts, self.world, self.rank, self.d_result, stream)
         return ShardResult(self.d_count, self.d_result, self.d_counts)
 
@@ -179,28 +220,27 @@ class ShardedDS:
         (module docstring).  Returns the number of outputs this rank holds
         at shard[0, ret); words past it are unspecified.  Host-synchronising
         (the plan needs the counts on the host)."""
-        counts = [int(c) for c in res.counts.tolist()]
+        with self._on(stream):
+            counts = [int(c) for c in res.counts.tolist()]  # host sync on the libds stream
         if self._sizes is None:
             mine = torch.tensor([shard.numel()], dtype=torch.int64, device=self.device)
             allsz = torch.zeros(self.world, dtype=torch.int64, device=self.device)
-            self._allgather(allsz, mine)
-            self._sizes = [int(x) for x in allsz.tolist()]
+            self._allgather(allsz, mine, stream)
+            with self._on(stream):
+                self._sizes = [int(x) for x in allsz.tolist()]
         plan = rebalance_plan(counts, self._sizes)
         me = self.rank
         for w in range(plan.waves):
-            ops = []
+            sends, recvs = [], []
             if plan.wave[me] == w:
-                for pc in plan.pieces:
-                    if pc.src == me:
-                        ops.append(dist.P2POp(dist.isend, shard[pc.src_lo:pc.src_lo + pc.count],
-                                              pc.dst, self.group))
-            for pc in plan.pieces:
-                if pc.dst == me and plan.wave[pc.src] == w:
-                    ops.append(dist.P2POp(dist.irecv, shard[pc.dst_lo:pc.dst_lo + pc.count],
-                                          pc.src, self.group))
-            if ops:
-                for req in dist.batch_isend_irecv(ops):
-                    req.wait()
+                sends = [(shard[pc.src_lo:pc.src_lo + pc.count], pc.dst) for pc in plan.pieces if pc.src == me]
+            recvs = [(shard[pc.dst_lo:pc.dst_lo + pc.count], pc.src) for pc in plan.pieces
+                     if pc.dst == me and plan.wave[pc.src] == w]
+            if sends or recvs:
+                # sends read, receives write the shard: both after the kernels
+                # before them on the stream, and the slide below after both
+                with self._on(stream):
+                    self.comm.exchange(sends, recvs)
             if plan.wave[me] == w and plan.shift[me] and plan.kept[me]:
                 self.local.slide(shard, counts[me], plan.shift[me], stream)
         return plan.final[me]
@@ -209,6 +249,6 @@ class ShardedDS:
         # Halo exchange before the slide (unique never changes a shard's last
         # word, but every rank must read its neighbour's value, R18).
         self.local.halo_entry(shard, self.d_entry, stream)
-        self._allgather(self.d_halo, self.d_entry)
+        self._allgather(self.d_halo, self.d_entry, stream)
         self.local.unique(shard, self.d_halo, self.rank, self.d_count, stream)
         return self._finish(stream)

@@ -78,9 +78,11 @@ def test_sharded_ds_world1_on_gpu():
 @pytest.mark.parametrize("G,fracs", [(2, [0.5, 0.5]), (4, [0.9, 0.1, 0.0, 1.0]), (8, [0.5] * 8),
                                      (3, [0.0, 0.7, 0.2])])
 def test_fake_shard_rebalance(G, fracs):
-    """Rebalance plan executed on one GPU: the NCCL send/recv of each wave
-    replaced by device copies between the fake shards, the gap closed by the
-    real ds_slide kernel.  Result: the single-array in-place compaction."""
+    """Rebalance plan executed on one GPU in one process: the NCCL send/recv of
+    each wave replaced by device copies between the fake shards, the gap
+    closed by the real ds_slide kernel.  Result: the single-array in-place
+    compaction.  (The product's ShardedDS.rebalance itself runs, with real
+    kernels and one process per rank, in tests/test_dist_multiproc_gpu.py.)"""
     from paper_conf_icpp_gomez_lunacshg15_b200.dist import rebalance_plan
     n = 2_000_003
     parts = []
