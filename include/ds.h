@@ -31,7 +31,12 @@
  *    the data) and one ticket/epoch word.  Calls that share a stream share it; calls on
  *    different streams may run concurrently.  ds_release_workspaces()
  *    frees it (call only when no libds kernel is in flight).
- *  - Thread-safe: host state is protected by a mutex.
+ *  - Thread-safe: host state (workspaces, launch parameters) is protected
+ *    by a mutex held only while a call validates and enqueues its kernels.
+ *    Every blocking call reads its count through a count word of its own
+ *    (taken from a per-device pool), and its read-back and stream
+ *    synchronisation run without the mutex, so concurrent blocking calls
+ *    never share a count and do not stall other threads' calls.
  */
 #ifndef LIBDS_DS_H
 #define LIBDS_DS_H

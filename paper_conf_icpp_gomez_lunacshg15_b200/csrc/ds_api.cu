@@ -10,6 +10,7 @@
 #include <mutex>
 #include <string>
 #include <utility>
+#include <vector>
 
 #include "ds.h"
 #include "ds_device.cuh"
@@ -24,6 +25,17 @@ constexpr uint64_t kResetEvery = 1ull << 25;         // zero statuses before the
 
 std::mutex g_mu;
 std::map<std::pair<int, uintptr_t>, ds::Workspace> g_ws;
+
+// Count words of the blocking forms: each call takes its own (device word,
+// pinned host mirror) pair from a per-device pool, so concurrent blocking
+// calls never share a count, and the read-back + stream sync run without
+// the lock (other threads' asynchronous calls are not stalled by it).
+struct CountSlot {
+    uint64_t* d = nullptr;
+    uint64_t* h = nullptr;
+};
+std::map<int, std::vector<CountSlot>> g_count_pool;  // free slots per device (g_mu)
+std::vector<std::pair<int, CountSlot>> g_count_all;   // every slot ever made (release)
 std::atomic<uint64_t> g_launches{0};
 std::atomic<uint64_t*> g_trace{nullptr};
 std::atomic<size_t> g_trace_cap{0};
@@ -43,17 +55,17 @@ ds_status get_workspace(size_t tiles, cudaStream_t s, ds::Workspace** out) {
     if (e != cudaSuccess) return fail(e, "cudaGetDevice");
     ds::Workspace& ws = g_ws[{dev, reinterpret_cast<uintptr_t>(s)}];
     if (!ws.ctrl) {
-        // ctrl = {epoch 1, ticket 0}; d_count lives right after it.
-        if ((e = cudaMalloc(&ws.ctrl, 2 * sizeof(uint64_t))) != cudaSuccess) {
-            ws.ctrl = nullptr;
+        // ctrl = {epoch 1, ticket 0}.  Nothing is kept unless every step succeeds,
+        // so a failed first call leaves no half-built workspace behind.
+        uint64_t* ctrl = nullptr;
+        if ((e = cudaMalloc(&ctrl, sizeof(uint64_t))) != cudaSuccess)
             return e == cudaErrorMemoryAllocation ? DS_ERROR_OUT_OF_MEMORY : fail(e, "cudaMalloc");
-        }
-        const uint64_t init[2] = {1ull << 32, 0};
-        if ((e = cudaMemcpy(ws.ctrl, init, sizeof(init), cudaMemcpyHostToDevice)) != cudaSuccess)
+        const uint64_t init = 1ull << 32;
+        if ((e = cudaMemcpy(ctrl, &init, sizeof(init), cudaMemcpyHostToDevice)) != cudaSuccess) {
+            cudaFree(ctrl);
             return fail(e, "cudaMemcpy");
-        ws.d_count = ws.ctrl + 1;
-        if ((e = cudaMallocHost(&ws.h_count, sizeof(uint64_t))) != cudaSuccess)
-            return fail(e, "cudaMallocHost");
+        }
+        ws.ctrl = ctrl;
     }
     if (ws.cap_tiles < tiles) {
         if (ws.status) {
@@ -80,6 +92,48 @@ ds_status get_workspace(size_t tiles, cudaStream_t s, ds::Workspace** out) {
     ws.launches++;
     *out = &ws;
     return DS_SUCCESS;
+}
+
+// Caller holds g_mu.
+ds_status take_count_slot(CountSlot* out) {
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return fail(e, "cudaGetDevice");
+    std::vector<CountSlot>& pool = g_count_pool[dev];
+    if (!pool.empty()) {
+        *out = pool.back();
+        pool.pop_back();
+        return DS_SUCCESS;
+    }
+    CountSlot c;
+    if ((e = cudaMalloc(&c.d, sizeof(uint64_t))) != cudaSuccess)
+        return e == cudaErrorMemoryAllocation ? DS_ERROR_OUT_OF_MEMORY : fail(e, "cudaMalloc");
+    if ((e = cudaMallocHost(&c.h, sizeof(uint64_t))) != cudaSuccess) {
+        cudaFree(c.d);
+        return e == cudaErrorMemoryAllocation ? DS_ERROR_OUT_OF_MEMORY : fail(e, "cudaMallocHost");
+    }
+    g_count_all.push_back({dev, c});
+    *out = c;
+    return DS_SUCCESS;
+}
+
+void give_count_slot(const CountSlot& c) {
+    std::lock_guard<std::mutex> lock(g_mu);
+    for (const auto& kv : g_count_all)
+        if (kv.second.d == c.d) {
+            g_count_pool[kv.first].push_back(c);
+            return;
+        }
+}
+
+// Reads a blocking call's count back (legacy default stream) without the lock.
+ds_status read_count(const CountSlot& c, size_t* out_n) {
+    cudaError_t e = cudaMemcpyAsync(c.h, c.d, sizeof(uint64_t), cudaMemcpyDeviceToHost, nullptr);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(nullptr);
+    ds_status st = e == cudaSuccess ? DS_SUCCESS : fail(e, "count read-back");
+    if (st == DS_SUCCESS) *out_n = size_t(*c.h);
+    give_count_slot(c);
+    return st;
 }
 
 ds_status run_irregular(const ds::IrregArgs& a, cudaStream_t s) {
@@ -116,20 +170,25 @@ ds_status irregular_blocking(ds::IrregArgs a, size_t* out_n) {
         *out_n = 0;
         return DS_SUCCESS;
     }
-    std::lock_guard<std::mutex> lock(g_mu);
-    cudaStream_t s = nullptr;
-    ds::Workspace* ws = nullptr;
-    ds_status st = get_workspace(ds::irregular_tiles(a), s, &ws);
-    if (st != DS_SUCCESS) return st;
-    a.d_out_n = ws->d_count;
-    cudaError_t e = ds::launch_irregular(a, *ws, s);
-    if (e != cudaSuccess) return fail(e, "irregular kernel launch");
-    if ((e = cudaMemcpyAsync(ws->h_count, ws->d_count, sizeof(uint64_t), cudaMemcpyDeviceToHost, s)) !=
-        cudaSuccess)
-        return fail(e, "cudaMemcpyAsync");
-    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return fail(e, "cudaStreamSynchronize");
-    *out_n = size_t(*ws->h_count);
-    return DS_SUCCESS;
+    CountSlot slot;
+    ds_status st;
+    {
+        std::lock_guard<std::mutex> lock(g_mu);
+        st = take_count_slot(&slot);
+        if (st != DS_SUCCESS) return st;
+        ds::Workspace* ws = nullptr;
+        st = get_workspace(ds::irregular_tiles(a), nullptr, &ws);
+        if (st == DS_SUCCESS) {
+            a.d_out_n = slot.d;
+            cudaError_t e = ds::launch_irregular(a, *ws, nullptr);
+            if (e != cudaSuccess) st = fail(e, "irregular kernel launch");
+        }
+    }
+    if (st != DS_SUCCESS) {
+        give_count_slot(slot);
+        return st;
+    }
+    return read_count(slot, out_n);
 }
 
 ds_status run_regular(const ds::RegArgs& a, cudaStream_t s);
@@ -441,27 +500,20 @@ ds_status ds_partition(void* ptr, size_t n, int predicate_id, void* aux, size_t*
         *out_n_true = 0;
         return DS_SUCCESS;
     }
-    uint64_t* d_cnt = nullptr;
-    uint64_t* h_cnt = nullptr;
+    // The true count goes to this call's own count word: the DS pass writes it
+    // and the tail copy reads it, so no other call may share it.
+    CountSlot slot;
     {
         std::lock_guard<std::mutex> lock(g_mu);
-        ds::Workspace* ws = nullptr;
-        st = get_workspace(ds::irregular_tiles(ds::IrregArgs{static_cast<uint32_t*>(ptr), n,
-                                                             ds::IrregOp::Select, 0, 0, nullptr, 0, nullptr}),
-                           nullptr, &ws);
+        st = take_count_slot(&slot);
         if (st != DS_SUCCESS) return st;
-        ws->launches--;  // only reserving the count words here
-        d_cnt = ws->d_count;
-        h_cnt = ws->h_count;
     }
-    st = ds_partition_ex(ptr, n, predicate_id, 0u, aux, d_cnt, nullptr);
-    if (st != DS_SUCCESS) return st;
-    std::lock_guard<std::mutex> lock(g_mu);
-    cudaError_t e = cudaMemcpyAsync(h_cnt, d_cnt, sizeof(uint64_t), cudaMemcpyDeviceToHost, nullptr);
-    if (e != cudaSuccess) return fail(e, "cudaMemcpyAsync");
-    if ((e = cudaStreamSynchronize(nullptr)) != cudaSuccess) return fail(e, "cudaStreamSynchronize");
-    *out_n_true = size_t(*h_cnt);
-    return DS_SUCCESS;
+    st = ds_partition_ex(ptr, n, predicate_id, 0u, aux, slot.d, nullptr);
+    if (st != DS_SUCCESS) {
+        give_count_slot(slot);
+        return st;
+    }
+    return read_count(slot, out_n_true);
 }
 
 ds_status ds_halo_entry(const void* ptr, size_t n, uint64_t* d_entry, ds_stream_t stream) {
@@ -551,9 +603,16 @@ ds_status ds_release_workspaces(void) {
         cudaDeviceSynchronize();
         if (ws.status) cudaFree(ws.status);
         if (ws.ctrl) cudaFree(ws.ctrl);
-        if (ws.h_count) cudaFreeHost(ws.h_count);
     }
     g_ws.clear();
+    for (auto& kv : g_count_all) {
+        if (cudaSetDevice(kv.first) != cudaSuccess) continue;
+        cudaDeviceSynchronize();
+        cudaFree(kv.second.d);
+        cudaFreeHost(kv.second.h);
+    }
+    g_count_all.clear();
+    g_count_pool.clear();
     cudaSetDevice(cur);
     return st;
 }

@@ -13,9 +13,7 @@ namespace ds {
 struct Workspace {
     uint64_t* status = nullptr;  // [cap_tiles]
     size_t cap_tiles = 0;
-    uint64_t* ctrl = nullptr;    // {epoch:32 | ticket:32}; device_count follows
-    uint64_t* d_count = nullptr; // blocking forms' device-side out_n
-    uint64_t* h_count = nullptr; // pinned host mirror of d_count
+    uint64_t* ctrl = nullptr;    // {epoch:32 | ticket:32}
     uint64_t launches = 0;       // launches since the status array was zeroed
 };
 

@@ -58,7 +58,89 @@ def main(reps):
                 libds.ds_unpad_ex(a, R, NC, C, 4, None)
                 torch.cuda.synchronize()
                 assert np.array_equal(u32(a), exp), ("unpad-back", rep, R, C, NC)
+        _more(rep, d_n)
     print(f"stress OK: {reps} reps with {libds.LIB_PATH}")
+
+
+def _dev(host_u32, mis):
+    """Device copy of host words starting `mis` words past a 16-byte boundary
+    (+ the tensor that owns the memory)."""
+    t = torch.zeros(host_u32.size + 8, dtype=torch.int32, device="cuda")
+    t[mis:mis + host_u32.size] = torch.from_numpy(host_u32.view(np.int32))
+    return t, t[mis:mis + host_u32.size]
+
+
+def _more(rep, d_n):
+    """The other kernel paths under the same reordering: partition (in place
+    through aux, and out of place), out-of-place select, 8-byte elements,
+    byte-granular pad/unpad, and ds_slide, at misaligned pointer phases."""
+    mis = rep % 4
+    n = 300_007 + rep
+    f = [0.0, 0.3, 0.5, 0.97, 1.0][rep % 5]
+    t = dsgen.select_threshold(f) & 0xFFFFFFFF
+    host = dsgen.select_input(n, 3000 + rep).numpy().view(np.uint32).copy()
+    # partition in place through aux
+    own, a = _dev(host, mis)
+    aown, aux = _dev(np.zeros(n, dtype=np.uint32), (mis + 1) % 4)
+    exp = host.copy()
+    m = oracle.partition(exp, oracle.PRED_I32_GT, t)
+    libds.ds_partition_ex(a, n, libds.DS_PRED_I32_GT, t, aux, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == m and np.array_equal(u32(a), exp), ("partition", rep)
+    # partition_copy and select_copy (out of place)
+    own, a = _dev(host, mis)
+    town, ot = _dev(np.zeros(n, dtype=np.uint32), (mis + 2) % 4)
+    fown, of = _dev(np.zeros(n, dtype=np.uint32), (mis + 3) % 4)
+    keep = (host.view(np.int32) > np.int32(t if t < 2**31 else t - 2**32))
+    libds.ds_partition_copy_ex(a, n, libds.DS_PRED_I32_GT, t, ot, of, d_n, None)
+    torch.cuda.synchronize()
+    k = int(keep.sum())
+    assert int(d_n.item()) == k, ("partition_copy count", rep)
+    assert np.array_equal(u32(ot)[:k], host[keep]) and np.array_equal(u32(of)[:n - k], host[~keep])
+    kept = oracle.select_copy(host, oracle.PRED_I32_GT, t)
+    libds.ds_select_copy_ex(a, n, libds.DS_PRED_I32_GT, t, ot, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == kept.size and np.array_equal(u32(ot)[:kept.size], kept), ("select_copy", rep)
+    # 8-byte elements
+    rng = np.random.default_rng(rep)
+    h64 = np.where(rng.random(n // 2) < f, rng.integers(1, 2**63, n // 2, dtype=np.int64), 0).view(np.uint64)
+    own, a = _dev(h64.view(np.uint32), 2 * (rep % 2))
+    exp = h64.copy()
+    m = oracle.compact64(exp, 0)
+    libds.ds_compact64_ex(a, h64.size, 0, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == m and np.array_equal(u32(a).view(np.uint64), exp), ("compact64", rep)
+    runs = np.repeat(rng.integers(0, 3, n // 2, dtype=np.int64), 3)[:n // 2].view(np.uint64)
+    own, a = _dev(runs.view(np.uint32), 2 * (rep % 2))
+    exp = runs.copy()
+    m = oracle.unique64(exp)
+    libds.ds_unique64_ex(a, runs.size, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == m and np.array_equal(u32(a).view(np.uint64), exp), ("unique64", rep)
+    # byte-granular pad / unpad (rows not whole words)
+    for (R, C, NC, eb) in ((2000, 999, 1003, 1), (700, 1501, 1510, 2)):
+        hb = rng.integers(0, 256, R * NC * eb, dtype=np.uint8)
+        tb = torch.zeros(hb.size + 64, dtype=torch.uint8, device="cuda")
+        off = (rep * eb) % 16
+        tb[off:off + hb.size] = torch.from_numpy(hb)
+        view = tb[off:off + hb.size]
+        exp = hb.copy()
+        oracle.pad(exp, R, C, NC, eb)
+        libds.ds_pad_ex(view, R, C, NC, eb, None, None)
+        torch.cuda.synchronize()
+        assert np.array_equal(view.cpu().numpy(), exp), ("pad bytes", rep, eb)
+        oracle.unpad(exp, R, NC, C, eb)
+        libds.ds_unpad_ex(view, R, NC, C, eb, None)
+        torch.cuda.synchronize()
+        assert np.array_equal(view.cpu().numpy(), exp), ("unpad bytes", rep, eb)
+    # slide
+    for shift in (1, 8195, 100_003):
+        own, a = _dev(host, mis)
+        exp = host.copy()
+        oracle.slide(exp, n, shift, 4)
+        libds.ds_slide_ex(a, n, shift, 4, None)
+        torch.cuda.synchronize()
+        assert np.array_equal(u32(a), exp), ("slide", rep, shift)
 
 
 if __name__ == "__main__":

@@ -625,3 +625,51 @@ def test_sub_word_unpad_large_drop_slow_path():
         oracle.unpad(exp, R, C, NC, eb)
         libds.ds_unpad(buf.ptr, R, C, NC, eb)
         buf.check(exp, f"unpad slow R={R} C={C} NC={NC} eb={eb}")
+
+
+# ------------------------------------------------------------ host threads
+def test_blocking_calls_from_threads():
+    """Blocking compact / unique / partition from 6 host threads at once (the
+    ctypes calls drop the GIL): every call gets its own count word, so each
+    result matches the oracle (partition's shared count)."""
+    import threading
+    n = 600_011
+    jobs = []
+    for j in range(6):
+        a = _u32(dsgen.select_input(n, 900 + j))
+        jobs.append(a)
+    results = [None] * len(jobs)
+
+    def work(j):
+        a = jobs[j]
+        t = dsgen.select_threshold(0.2 + 0.1 * j) & 0xFFFFFFFF
+        out = []
+        for rep in range(4):
+            buf = DevBuf(a, (j + rep) % 4)
+            exp = buf.host_region()
+            if (j + rep) % 3 == 0:
+                m_exp = oracle.compact(exp, int(a[7]))
+                m = libds.ds_compact(buf.ptr, n, int(a[7]))
+            elif (j + rep) % 3 == 1:
+                m_exp = oracle.unique(exp)
+                m = libds.ds_unique(buf.ptr, n)
+            else:
+                exp_p = exp.copy()
+                m_exp = oracle.partition(exp_p, oracle.PRED_I32_GT, 0)
+                exp = exp_p
+                aux = torch.empty(n, dtype=torch.int32, device="cuda")
+                m = libds.ds_partition(buf.ptr, n, libds.DS_PRED_I32_GT, aux)
+            out.append((m, m_exp, buf, exp))
+        results[j] = out
+
+    with torch.cuda.device(0):
+        threads = [threading.Thread(target=work, args=(j,)) for j in range(len(jobs))]
+        for th in threads:
+            th.start()
+        for th in threads:
+            th.join()
+    for j, out in enumerate(results):
+        assert out is not None, j
+        for m, m_exp, buf, exp in out:
+            assert m == m_exp
+            buf.assert_equals(exp, f"thread {j}")
