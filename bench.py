@@ -15,8 +15,14 @@ reading a 512 MiB buffer.  value = sum over ranks of 4*(n_r + out_r) bytes /
 max-over-ranks device time of the step.
 
 rows (N == 1 only): the other BASELINE configs through the same C ABI --
-C1 compact 1M, C2 pad / unpad 4000x3990 <-> 4000, C3 select and unique on
-256M over f = 0..1, C4 compact 1G float32 at 10/50/90 %.
+C1 compact 1M (flushed and L2-hot kernel time, blocking-API wall time, the
+oracle in seconds), C2 pad / unpad 4000x3990 <-> 4000, pad / unpad at >= 256M
+elements (16384x16383 <-> 16384 in f32 and in 8-byte elements) and the Table-I
+shape 12000x11999 -> 12000, C3 select and unique on 256M over f = 0..1, C4
+compact 1G float32 at 10/50/90 %, partition, out-of-place select, int64
+compaction, 1- and 2-byte pad/unpad.  Every time is the median of the reps,
+with min and p90 beside it; fractions are given of the measured copy peak
+(MEASURED_PEAKS.json) and of the nominal 8 TB/s.
 
 --impl reference: the CPU oracle (oracle/, sequential C, one core) on a
 bounded sample of the same workload, rank 0 only.
@@ -39,6 +45,17 @@ N_TOTAL = 1 << 32
 FRAC = 0.5
 SEED = 0xD5201500 + 16 * 4  # dsgen.seed_for(4): C5
 WORKLOAD = "C5: sharded in-place stream compaction of 4G int32 (2^32 words), 50% kept, remove_value 0"
+
+
+NOMINAL_HBM_GBS = 8000.0  # B200 HBM3e nominal (B200_PROFILING.md); the measured copy rate is the ceiling
+
+
+def summarize(ts_ms):
+    """median / min / p90 of a list of times (ms) -> microseconds."""
+    xs = sorted(ts_ms)
+    p90 = xs[min(len(xs) - 1, int(round(0.9 * (len(xs) - 1))))]
+    return {"us": round(statistics.median(xs) * 1e3, 2), "min_us": round(xs[0] * 1e3, 2),
+            "p90_us": round(p90 * 1e3, 2), "reps": len(xs)}
 
 
 def load_peaks():
@@ -106,7 +123,7 @@ class ClockSampler:
 
 
 def timed(fn, stream, restore=None, flush=None, reps=5, warmup=2):
-    """Median device time (ms) of fn() on `stream`, events around fn only."""
+    """Device times (ms, one per rep) of fn() on `stream`, events around fn only."""
     import torch
     ts = []
     for r in range(warmup + reps):
@@ -121,50 +138,105 @@ def timed(fn, stream, restore=None, flush=None, reps=5, warmup=2):
         b.synchronize()
         if r >= warmup:
             ts.append(a.elapsed_time(b))
-    return statistics.median(ts)
+    return ts
 
 
 def bench_rows(peak, flush):
     """The other BASELINE configs (rank 0, N == 1)."""
+    import numpy as np
     import torch
 
     import dsgen
+    import oracle
     from paper_conf_icpp_gomez_lunacshg15_b200 import libds
     s = torch.cuda.current_stream()
     d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
     rows = []
 
-    def row(op, cfg, ms, nbytes, extra=None):
-        gbs = nbytes / (ms * 1e-3) / 1e9
-        r = {"op": op, "config": cfg, "us": round(ms * 1e3, 2), "gbs": round(gbs, 1),
-             "frac": round(gbs / peak, 4)}
+    def row(op, cfg, ts, nbytes, extra=None, dram_bytes=None):
+        st = summarize(ts)
+        gbs = nbytes / (st["us"] * 1e-6) / 1e9
+        r = {"op": op, "config": cfg, **st, "gbs": round(gbs, 1), "frac": round(gbs / peak, 4),
+             "frac_nominal": round(gbs / NOMINAL_HBM_GBS, 4)}
+        if dram_bytes is not None and dram_bytes != nbytes:
+            # identity moves store nothing: the DRAM bytes the kernel must move
+            r["dram_bytes"] = dram_bytes
+            r["frac_dram"] = round(dram_bytes / (st["us"] * 1e-6) / 1e9 / peak, 4)
         if extra:
             r.update(extra)
         rows.append(r)
+        return r
 
     def irregular(op, name, src, call, reps=5):
         work = torch.empty_like(src)
-        ms = timed(lambda: call(work), s, restore=lambda: work.copy_(src), flush=flush, reps=reps)
+        ts = timed(lambda: call(work), s, restore=lambda: work.copy_(src), flush=flush, reps=reps)
         m = int(d_n.item())
-        row(op, name, ms, 4 * (src.numel() + m), {"n": src.numel(), "out_n": m})
+        n = src.numel()
+        # an in-place call that removes nothing is an identity move: every tile
+        # is skipped by the storers, only the reads reach DRAM (DESIGN.md §7)
+        row(op, name, ts, 4 * (n + m), {"n": n, "out_n": m}, dram_bytes=4 * n if m == n else None)
 
-    # C1: 1M int32 compaction, 50 %
+    def regular(op, name, src, call, nbytes, reps=5, restore_src=None):
+        work = torch.empty_like(src)
+        base = restore_src if restore_src is not None else src
+        ts = timed(lambda: call(work), s, restore=lambda: work.copy_(base), flush=flush, reps=reps)
+        row(op, name, ts, nbytes)
+
+    # C1: 1M int32 compaction, 50 %: kernel time flushed and L2-hot, the blocking
+    # call's wall time (launch + sync + D2H of out_n), and the oracle in seconds
     n = 1 << 20
     src = dsgen.compact_input(n, 0.5, dsgen.seed_for(0), device="cuda")
-    irregular("compact", "C1 1M int32 f=0.5", src,
-              lambda w: libds.ds_compact_ex(w, n, 0, d_n, None), reps=20)
+    work = torch.empty_like(src)
+    ts = timed(lambda: libds.ds_compact_ex(work, n, 0, d_n, None), s, restore=lambda: work.copy_(src),
+               flush=flush, reps=50)
+    m = int(d_n.item())
+    ts_hot = timed(lambda: libds.ds_compact_ex(work, n, 0, d_n, None), s, restore=lambda: work.copy_(src),
+                   reps=50)
+    wall = []
+    for r in range(53):
+        work.copy_(src)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        libds.ds_compact(work, n, 0)
+        if r >= 3:
+            wall.append((time.perf_counter() - t0) * 1e3)
+    host = src.cpu().numpy().view(np.uint32).copy()
+    ot = []
+    for _ in range(5):
+        hcopy = host.copy()
+        t0 = time.perf_counter()
+        oracle.compact(hcopy, 0)
+        ot.append(time.perf_counter() - t0)
+    row("compact", "C1 1M int32 f=0.5", ts, 4 * (n + m),
+        {"n": n, "out_n": m, "l2_hot": summarize(ts_hot), "blocking_wall": summarize(wall),
+         "oracle_s": round(statistics.median(ot), 6),
+         "note": "flushed: 512 MiB read between reps; l2_hot: input restored by a D2D copy only "
+                 "(it stays in L2); blocking_wall: ds_compact (legacy stream) incl. the D2H of out_n"})
+    del src, work
     # C2: pad 4000x3990 -> 4000 f32 and unpad back
     R, C, NC = 4000, 3990, 4000
     src = dsgen.matrix_input(R, C, NC, 4, kind="f32", device="cuda")
-    work = torch.empty_like(src)
-    ms = timed(lambda: libds.ds_pad_ex(work, R, C, NC, 4, None, None), s,
-               restore=lambda: work.copy_(src), flush=flush, reps=20)
-    row("pad", "C2 4000x3990->4000 f32", ms, 4 * (R * C + R * NC))
+    regular("pad", "C2 4000x3990->4000 f32", src, lambda w: libds.ds_pad_ex(w, R, C, NC, 4, None, None),
+            4 * (R * C + R * NC), reps=20)
     padded = src.clone()
     libds.ds_pad(padded, R, C, NC, 4)
-    ms = timed(lambda: libds.ds_unpad_ex(work, R, NC, C, 4, None), s,
-               restore=lambda: work.copy_(padded), flush=flush, reps=20)
-    row("unpad", "C2 4000x4000->3990 f32", ms, 4 * (2 * R * C))
+    regular("unpad", "C2 4000x4000->3990 f32", src, lambda w: libds.ds_unpad_ex(w, R, NC, C, 4, None),
+            4 * (2 * R * C), reps=20, restore_src=padded)
+    del src, padded
+    # Pad / unpad where the >= 70 % target applies (>= 256M elements): 16384 x
+    # 16383 <-> 16384 in f32 and in 8-byte elements (P:220, P:226), and the
+    # Table-I shape 12000 x 11999 -> 12000 (P:325)
+    for (R, C, NC, eb, tag) in ((16384, 16383, 16384, 4, "f32"), (16384, 16383, 16384, 8, "8-byte"),
+                                (12000, 11999, 12000, 4, "f32 Table I")):
+        src = dsgen.matrix_input(R, C, NC, eb, device="cuda")
+        regular("pad", f"{R}x{C}->{NC} {tag}", src, lambda w: libds.ds_pad_ex(w, R, C, NC, eb, None, None),
+                eb * (R * C + R * NC), reps=5)
+        padded = src.clone()
+        libds.ds_pad(padded, R, C, NC, eb)
+        regular("unpad", f"{R}x{NC}->{C} {tag}", src, lambda w: libds.ds_unpad_ex(w, R, NC, C, eb, None),
+                eb * 2 * R * C, reps=5, restore_src=padded)
+        del src, padded
+        torch.cuda.empty_cache()
     # C3: select (x > t) and unique, 256M int32, f = 0 .. 1
     n = 1 << 28
     src = dsgen.select_input(n, dsgen.seed_for(2), device="cuda")
@@ -172,13 +244,13 @@ def bench_rows(peak, flush):
         f = i / 10
         t = dsgen.select_threshold(f) & 0xFFFFFFFF
         irregular("select", f"C3 256M int32 x>t f={f:.1f}", src,
-                  lambda w, t=t: libds.ds_select_ex(w, n, libds.DS_PRED_I32_GT, t, d_n, None), reps=3)
+                  lambda w, t=t: libds.ds_select_ex(w, n, libds.DS_PRED_I32_GT, t, d_n, None), reps=5)
     del src
     for i in range(11):
         f = i / 10
         src = dsgen.unique_runs_input(n, f, dsgen.seed_for(2, 11 + i), device="cuda")
         irregular("unique", f"C3 256M int32 runs f={f:.1f}", src,
-                  lambda w: libds.ds_unique_ex(w, n, None, 0, d_n, None), reps=3)
+                  lambda w: libds.ds_unique_ex(w, n, None, 0, d_n, None), reps=5)
         del src
     # Partition (in place through an aux buffer) and out-of-place
     # select (Copy_if) on 256M int32 at 50 %
@@ -187,22 +259,22 @@ def bench_rows(peak, flush):
     t = dsgen.select_threshold(0.5) & 0xFFFFFFFF
     aux = torch.empty_like(src)
     work = torch.empty_like(src)
-    ms = timed(lambda: libds.ds_partition_ex(work, n, libds.DS_PRED_I32_GT, t, aux, d_n, None), s,
-               restore=lambda: work.copy_(src), flush=flush, reps=3)
+    ts = timed(lambda: libds.ds_partition_ex(work, n, libds.DS_PRED_I32_GT, t, aux, d_n, None), s,
+               restore=lambda: work.copy_(src), flush=flush, reps=5)
     m = int(d_n.item())
-    row("partition", "256M int32 x>t f=0.5 (in place, aux)", ms, 4 * (2 * n + 2 * (n - m)),
+    row("partition", "256M int32 x>t f=0.5 (in place, aux)", ts, 4 * (2 * n + 2 * (n - m)),
         {"n": n, "out_n": m, "bytes": "read n + write n_true in place + write/read/write n_false via aux"})
-    ms = timed(lambda: libds.ds_select_copy_ex(src, n, libds.DS_PRED_I32_GT, t, work, d_n, None), s,
-               flush=flush, reps=3)
+    ts = timed(lambda: libds.ds_select_copy_ex(src, n, libds.DS_PRED_I32_GT, t, work, d_n, None), s,
+               flush=flush, reps=5)
     m = int(d_n.item())
-    row("select_copy", "256M int32 x>t f=0.5 (out of place)", ms, 4 * (n + m), {"n": n, "out_n": m})
+    row("select_copy", "256M int32 x>t f=0.5 (out of place)", ts, 4 * (n + m), {"n": n, "out_n": m})
     del src, aux, work
     # C4: 1G float32 compaction at 10 / 50 / 90 %
     n = 1 << 30
     for f in (0.1, 0.5, 0.9):
         src = dsgen.compact_input(n, f, dsgen.seed_for(3, int(f * 10)), kind="f32", device="cuda")
         irregular("compact", f"C4 1G f32 f={f}", src,
-                  lambda w: libds.ds_compact_ex(w, n, 0, d_n, None), reps=3)
+                  lambda w: libds.ds_compact_ex(w, n, 0, d_n, None), reps=5)
         del src
     # 8(f)-3: 8-byte elements (int64 compaction, 256M elements = 2 GiB, 50 % kept)
     n = 1 << 28
@@ -210,24 +282,23 @@ def bench_rows(peak, flush):
     src = torch.where(dsgen._hi32(h) < dsgen.keep_threshold(0.5), h | 1, torch.zeros_like(h))
     del h
     work = torch.empty_like(src)
-    ms = timed(lambda: libds.ds_compact64_ex(work, n, 0, d_n, None), s, restore=lambda: work.copy_(src),
-               flush=flush, reps=3)
+    ts = timed(lambda: libds.ds_compact64_ex(work, n, 0, d_n, None), s, restore=lambda: work.copy_(src),
+               flush=flush, reps=5)
     m = int(d_n.item())
-    row("compact64", "256M int64 f=0.5 (8-byte elements)", ms, 8 * (n + m), {"n": n, "out_n": m})
+    row("compact64", "256M int64 f=0.5 (8-byte elements)", ts, 8 * (n + m), {"n": n, "out_n": m})
     del src, work
     # 8(f)-4: sub-word elements, C2 shape (byte-granular kernel for 1-byte rows of
-    # 3990 bytes; 2-byte rows are whole words and take the word kernel)
-    R, C, NC = 4000, 3990, 4000
-    for eb in (1, 2):
-        src = torch.randint(0, 256, (R * NC * eb,), dtype=torch.uint8, device="cuda")
-        work = torch.empty_like(src)
-        ms = timed(lambda: libds.ds_pad_ex(work, R, C, NC, eb, None, None), s,
-                   restore=lambda: work.copy_(src), flush=flush, reps=20)
-        row("pad", f"C2 shape {R}x{C}->{NC} eb={eb}", ms, eb * (R * C + R * NC))
-        ms = timed(lambda: libds.ds_unpad_ex(work, R, NC, C, eb, None), s,
-                   restore=lambda: work.copy_(src), flush=flush, reps=20)
-        row("unpad", f"C2 shape {R}x{NC}->{C} eb={eb}", ms, eb * 2 * R * C)
-        del src, work
+    # 3990 bytes; 2-byte rows are whole words and take the word kernel), and a
+    # >= 256M-element byte shape (16384 x 16383 -> 16384, 1-byte elements)
+    for (R, C, NC) in ((4000, 3990, 4000), (16384, 16383, 16384)):
+        for eb in ((1, 2) if R == 4000 else (1,)):
+            src = torch.randint(0, 256, (R * NC * eb,), dtype=torch.uint8, device="cuda")
+            reps = 20 if R == 4000 else 5
+            regular("pad", f"{R}x{C}->{NC} eb={eb}", src,
+                    lambda w: libds.ds_pad_ex(w, R, C, NC, eb, None, None), eb * (R * C + R * NC), reps=reps)
+            regular("unpad", f"{R}x{NC}->{C} eb={eb}", src,
+                    lambda w: libds.ds_unpad_ex(w, R, NC, C, eb, None), eb * 2 * R * C, reps=reps)
+            del src
     return rows
 
 
@@ -295,6 +366,9 @@ def run_libds(args):
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
+        # the driver reads NCCL's communicator-init lines (nRanks) from stderr
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         dist.init_process_group("nccl", device_id=dev)
     peak, peak_src = load_peaks()
 
@@ -351,22 +425,51 @@ def run_libds(args):
     barrier()
     launches = libds.ds_launch_count() - launches0
     clk = clocks.stop()
-    step_ms = sum(e[0].elapsed_time(e[2]) for e in evs)
-    kern_ms = sum(e[0].elapsed_time(e[1]) for e in evs) / args.steps
+    step_list = [e[0].elapsed_time(e[2]) for e in evs]
+    kern_list = [e[0].elapsed_time(e[1]) for e in evs]
+    coll_list = [e[1].elapsed_time(e[2]) for e in evs]
+    step_ms = sum(step_list)
+    kern_ms = sum(kern_list) / args.steps
+    coll_ms = sum(coll_list) / args.steps
     out_n = int(ds.d_count.item())
     total_out = int(ds.d_result[1].item())
     my_bytes = 4 * (n + out_n)
-    t = torch.tensor([step_ms, float(my_bytes)], dtype=torch.float64, device=dev)
+    # per-rank [step total, bytes, kernel ms/step, collective ms/step]; max / sum over ranks
+    t = torch.tensor([step_ms, float(my_bytes), kern_ms, coll_ms], dtype=torch.float64, device=dev)
     if world > 1:
-        tmax = t[:1].clone()
-        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
-        tsum = t[1:].clone()
-        dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
-        step_ms_max, all_bytes = float(tmax.item()), float(tsum.item())
+        allt = torch.zeros(world * 4, dtype=torch.float64, device=dev)
+        dist.all_gather_into_tensor(allt, t)
+        per_rank = allt.view(world, 4).tolist()
     else:
-        step_ms_max, all_bytes = step_ms, float(my_bytes)
+        per_rank = [t.tolist()]
+    step_ms_max = max(r[0] for r in per_rank)
+    all_bytes = sum(r[1] for r in per_rank)
     ms_per_step = step_ms_max / args.steps
     value = all_bytes / (ms_per_step * 1e-3) / 1e9
+
+    # ---- optional rebalance leg (8(f)-1), timed separately after a compact step
+    rebal = None
+    if args.rebalance:
+        rts = []
+        for i in range(1 + max(1, args.steps // 4)):
+            work.copy_(pristine)
+            barrier()
+            res = ds.compact(work, 0, stream=stream)
+            barrier()
+            t0 = torch.cuda.Event(enable_timing=True)
+            t1 = torch.cuda.Event(enable_timing=True)
+            t0.record(stream)
+            held = ds.rebalance(work, res, stream=stream)
+            t1.record(stream)
+            barrier()
+            if i > 0:
+                rts.append(t0.elapsed_time(t1))
+        mine = torch.tensor([statistics.median(rts)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(mine, op=dist.ReduceOp.MAX)
+        rebal = {"ms": round(float(mine.item()), 4), "held_rank0": held,
+                 "note": "ShardedDS.rebalance after the compact step: wave-scheduled NCCL send/recv of "
+                         "the pieces + ds_slide; host-synchronising plan; max over ranks"}
 
     # ---- e2e through the public API with host buffers (pinned), copies inside the timing.
     # The shard goes through in E2E_CHUNKS pieces on three streams so that the
@@ -454,6 +557,7 @@ def run_libds(args):
         kbytes = 4 * (n + out_n)
         achieved = kbytes / (kern_ms * 1e-3) / 1e9
         traffic = load_ncu_traffic()
+        step_stats = summarize(step_list)
         line = {
             "metric": METRIC, "value": round(value, 1), "unit": "GB/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
@@ -467,9 +571,17 @@ def run_libds(args):
                        "restore": "pristine shard restored by a D2D copy between steps, outside the events",
                        "step": "ds_compact_ex + NCCL all-gather of counts + ds_shard_offsets"},
             "frac_of_peak": round(value / world / peak, 4),
+            "frac_of_nominal": round(value / world / NOMINAL_HBM_GBS, 4),
             "elems_per_s": round(N_TOTAL / (ms_per_step * 1e-3), 1),
+            "step_stats_rank0": step_stats,
+            "per_rank": [{"rank": r, "step_ms": round(x[0] / args.steps, 4), "kernel_ms": round(x[2], 4),
+                          "collective_ms": round(x[3], 4)} for r, x in enumerate(per_rank)],
+            "kernel_ms_max": round(max(x[2] for x in per_rank), 4),
+            "collective_ms_max": round(max(x[3] for x in per_rank), 4),
             "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                          "frac": round(achieved / peak, 4), "traffic": traffic,
+                         "frac_nominal": round(achieved / NOMINAL_HBM_GBS, 4),
+                         "kernel_stats": summarize(kern_list),
                          "kernel": "irregular_kernel<OpCompact> (rank 0)", "peak_source": peak_src,
                          "kernel_ms": round(kern_ms, 4),
                          "algorithmic_bytes_per_launch": kbytes},
@@ -477,6 +589,8 @@ def run_libds(args):
         }
         if e2e:
             line["e2e"] = e2e
+        if rebal:
+            line["rebalance"] = rebal
         if cpu:
             line["cpu_baseline"] = cpu
         if rows:
@@ -498,6 +612,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--e2e-chunks", type=int, default=32)
+    ap.add_argument("--rebalance", action="store_true", help="also time ShardedDS.rebalance (8(f)-1)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "libds" and not os.environ.get("DS_BENCH_ALLOW_SHORT"):
         args.warmup = 3

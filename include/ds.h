@@ -19,6 +19,19 @@
  *    DS_ERROR_INVALID_VALUE / DS_ERROR_UNSUPPORTED return the buffer and
  *    the output count are untouched.  DS_ERROR_CUDA means a CUDA call
  *    failed after launch; the buffer content is then undefined (in place).
+ *  - Reads: the kernels stage data with 16-byte TMA bulk copies.  A copy
+ *    may start up to 12 bytes BEFORE ptr (the words before ptr in ptr's own
+ *    16-byte-aligned chunk, which lie in the same allocation because device
+ *    allocations start 256-byte aligned); their values are never used or
+ *    written.  Nothing past the end of the caller's buffer is read: the last
+ *    partial chunk of an array is loaded word by word (compact / select /
+ *    unique / partition), and a pad / unpad / slide tile whose chunk would
+ *    pass the end of the buffer (pad: rows*new_cols elements, unpad and
+ *    slide: the sources) is gathered element by element.  Checked by
+ *    compute-sanitizer memcheck with arrays that end at their allocation's
+ *    end (tests/test_sanitizer_gpu.py).
+ *  - Writes: only the output positions of the operation (and the fill cells
+ *    of pad); never a word outside them.
  *  - Kept outputs are stable.  Words in [out_n, n) (compact/select/
  *    unique) and in [rows*new_cols, rows*cols) elements (unpad) are left
  *    exactly as they were (R5).

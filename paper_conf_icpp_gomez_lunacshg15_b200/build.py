@@ -8,6 +8,8 @@ its own so Python never mistakes it for an extension module).  Variants:
   release : -O3 -lineinfo                            -> libds.so
   stress  : -DDS_DEBUG_DELAY (random per-CTA delays) -> libds_stress.so
   strict  : -DDS_STRICT_ORDER (release/acquire status ordering) -> libds_strict.so
+  spincap : -DDS_SPIN_CAP_NS (waits trap after 2 s: failure detection) -> libds_spincap.so
+  hang    : spincap + -DDS_DEBUG_DROP_TILE=5 (a lost tile; test only) -> libds_hang.so
 The CUDA runtime is linked statically so the library does not depend on
 which libcudart the host process (torch) has loaded.
 """
@@ -30,6 +32,10 @@ VARIANTS = {
     "release": ("libds.so", []),
     "stress": ("libds_stress.so", ["-DDS_DEBUG_DELAY=1"]),
     "strict": ("libds_strict.so", ["-DDS_STRICT_ORDER=1"]),
+    # failure detection: every wait traps after 2 s (no false positive expected)
+    "spincap": ("libds_spincap.so", ["-DDS_SPIN_CAP_NS=2000000000ull"]),
+    # the same with tile 5 of every irregular launch never publishing (test only)
+    "hang": ("libds_hang.so", ["-DDS_SPIN_CAP_NS=200000000ull", "-DDS_DEBUG_DROP_TILE=5u"]),
 }
 
 

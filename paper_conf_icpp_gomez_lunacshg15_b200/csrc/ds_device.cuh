@@ -17,6 +17,7 @@
 #pragma once
 
 #include <cstdint>
+#include <cstdio>
 
 namespace ds {
 
@@ -155,10 +156,39 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
 }
+// Failure detection: with -DDS_SPIN_CAP_NS=t every wait loop of
+// the kernels gives up after t ns of waiting and traps (printing where), so a
+// lost publication (a bug, or DS_DEBUG_DROP_TILE) ends the launch with a CUDA
+// error that the API reports as DS_ERROR_CUDA instead of hanging the process.
+// Compiled out of the release library.
+struct SpinGuard {
+#ifdef DS_SPIN_CAP_NS
+    uint64_t t0 = 0;
+    __device__ __forceinline__ void check(const char* where) {
+        uint64_t now;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now));
+        if (t0 == 0) t0 = now;
+        else if (now - t0 > uint64_t(DS_SPIN_CAP_NS)) {
+            printf("libds: wait in %s exceeded DS_SPIN_CAP_NS (block %d thread %d)\n", where, blockIdx.x,
+                   threadIdx.x);
+            __trap();
+        }
+    }
+#else
+    __device__ __forceinline__ void check(const char*) {}
+#endif
+};
+
 // Blocking wait for the phase with the given parity.  The suspend-time hint
 // lets the hardware park the warp until the phase completes instead of
 // re-issuing try_wait in a tight loop.
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity, uint32_t hint_ns);
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+#ifdef DS_SPIN_CAP_NS
+    SpinGuard g;
+    while (!mbar_try_wait(bar, parity, 100000u)) g.check("mbarrier wait");
+    return;
+#endif
 #ifdef DS_MBAR_SPIN
     asm volatile(
         "{\n"

@@ -252,6 +252,13 @@ __device__ __forceinline__ bool halo_prev(const IrregParams& p, uint32_t& prev) 
 #endif
 constexpr uint32_t kPollMinNs = DS_IRR_POLL_MIN;   // first back-off
 constexpr uint32_t kPollMaxNs = DS_IRR_POLL_MAX;   // back-off cap
+// Fault injection for the failure-detection test only: tile DS_DEBUG_DROP_TILE
+// never publishes its status (as if its CTA were lost), so every later tile's
+// look-back waits forever; built together with DS_SPIN_CAP_NS.
+#ifndef DS_DEBUG_DROP_TILE
+#define DS_DEBUG_DROP_TILE 0xffffffffu
+#endif
+constexpr uint32_t kDropTile = DS_DEBUG_DROP_TILE;
 #ifndef DS_IRR_LATE_LB
 #define DS_IRR_LATE_LB 1
 #endif
@@ -263,6 +270,7 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
     uint32_t rounds = 0, polls = 0;
     int64_t base = int64_t(tile) - 1;
     uint32_t ns = kPollMinNs;
+    SpinGuard guard;
     while (true) {
         int64_t idx = base - lane;
         uint64_t s = idx >= 0 ? ld_relaxed_gpu(status_ptr(status, idx)) : make_status(kStateIncl, epoch, 0);
@@ -274,6 +282,7 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
             L = inclm ? uint32_t(__ffs(inclm) - 1) : 32u;
             const bool need = uint32_t(lane) <= L;  // every lane up to the nearest INCL
             if (!__any_sync(kFull, need && !ok)) break;
+            guard.check("irregular look-back");
             __nanosleep(ns);
             ns = ns < kPollMaxNs ? ns * 2 : kPollMaxNs;
             ++polls;
@@ -402,7 +411,9 @@ constexpr uint32_t kEndPollNs = DS_IRR_END_POLL_NS;
 __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
                                                  const volatile uint32_t* s_end, uint32_t k) {
     if (DS_IRR_TESTWAIT && mbar_test_wait(bar, parity)) return true;  // no suspension if already complete
+    SpinGuard guard;
     while (true) {
+        guard.check("irregular end-aware wait");
         if (mbar_try_wait(bar, parity, kEndPollNs)) return true;
         // Strictly beyond the end marker: the position holding the marker
         // itself still gets its arrival and must pass it on.
@@ -480,7 +491,11 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             // any free input stage (a tile compacted into the ring frees its stage at
             // once, one compacted in place only once stored)
             uint32_t m;
-            while ((m = ld_acquire_cta_smem(&s_stages)) == 0u) __nanosleep(32);
+            SpinGuard guard;
+            while ((m = ld_acquire_cta_smem(&s_stages)) == 0u) {
+                guard.check("irregular producer stage wait");
+                __nanosleep(32);
+            }
             const uint32_t s = __ffs(m) - 1;
             atomicAnd(&s_stages, ~(1u << s));
             uint32_t* stage = smem + s * kStageWords;
@@ -509,18 +524,23 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             trace_event(p.trace, t, 7, smid());
             debug_delay(t, 0);
             const uint64_t tb = uint64_t(t) * kT;
-            uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
-            // The copy covers whole 16-byte chunks: it may read up to 12 bytes past
-            // the array end and the (lo) words before ptr, inside the same chunks
-            // (include/ds.h, "Reads").
-            end = (end + 3) & ~3ull;
+            const uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
+            // The bulk copy covers whole 16-byte chunks from the tile's aligned
+            // start: tile 0 also reads the (lo) words before ptr, which share
+            // ptr's 16-byte chunk.  It stops at the last whole chunk of the
+            // array; the 1..3 words after it (last tile only) are loaded by this
+            // thread, so nothing past the array's end is read (include/ds.h).
+            const uint64_t end16 = end & ~3ull;
             // Unique also needs the word before the tile: one copy starting kPre
             // words early (measured faster than a separate 16-byte copy).
             const uint64_t beg = (Op::kUnique && t > 0) ? tb - kPre : tb;
-            const uint32_t bytes = uint32_t(end - beg) * 4u;
+            uint32_t* const dst = stage + kPre - (tb - beg);
+            for (uint64_t w = end16 > beg ? end16 : beg; w < end; ++w)
+                dst[w - beg] = ldg_stream(p.abase + w);  // before the arrival that publishes the stage
+            const uint32_t bytes = end16 > beg ? uint32_t(end16 - beg) * 4u : 0u;
             fence_proxy_async_smem();
             mbar_arrive_expect_tx(&bar_loaded[o], bytes);
-            bulk_g2s(stage + kPre - (tb - beg), p.abase + beg, bytes, &bar_loaded[o]);
+            if (bytes) bulk_g2s(dst, p.abase + beg, bytes, &bar_loaded[o]);
         }
     } else if (warp < kRankWarps) {
         // ------------------------------------------------ ranker warps
@@ -667,7 +687,8 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 // (a relaxed status store).
                 meta[o].total = total;
                 debug_delay(t, 1);
-                publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
+                if (t != kDropTile)
+                    publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));
                 trace_event(p.trace, t, 2, globaltimer());
                 mbar_arrive(&bar_counted[o]);
             }
@@ -684,7 +705,10 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             if (k > 0) {
                 if (kRankGroups > 1) {
                     if (lane == 0)
-                        while (ld_acquire_cta_smem(&s_alloc) < k) __nanosleep(32);
+                        for (SpinGuard guard; ld_acquire_cta_smem(&s_alloc) < k;) {
+                            guard.check("irregular ring allocation order");
+                            __nanosleep(32);
+                        }
                     __syncwarp();
                 }
                 const SlotMeta& pm = meta[(k + kSlots - 1) % kSlots];
@@ -770,7 +794,8 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint64_t excl = t > 0 ? lookback(p.status, t, epoch, lane, p.trace) : 0ull;
             if (!kLateLookback) mbar_wait(&bar_counted[o], use & 1);  // the tile's aggregate is published
             const uint32_t total = meta[o].total;
-            if (lane == 0 && t > 0) publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
+            if (lane == 0 && t > 0 && t != kDropTile)
+                publish_status(status_ptr(p.status, t), make_status(kStateIncl, epoch, excl + total));
             mbar_wait(&bar_ranked[o], use & 1);  // the compacted tile is in the ring
             if (lane == 0) {
                 trace_event(p.trace, t, 4, globaltimer());

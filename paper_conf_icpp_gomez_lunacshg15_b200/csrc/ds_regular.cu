@@ -92,9 +92,13 @@ __device__ void tile_geometry(const RegParams& p, int64_t k, TileGeom& g) {
     }
     g.slo = slo;
     g.span = shi >= slo ? shi - slo + 1 : 0;
-    g.sb = (slo + mis) & ~int64_t(3);
-    const int64_t se = (slo + mis + g.span + 3) & ~int64_t(3);  // may pass the end by <= 3 words
-    g.fast = (se - g.sb) <= STAGE;
+    g.sb = (slo + mis) & ~int64_t(3);  // lead words: inside the 16-byte chunk holding slo
+    const int64_t se = (slo + mis + g.span + 3) & ~int64_t(3);
+    // The bulk copy covers whole 16-byte chunks; a chunk that would pass the end
+    // of the caller's buffer (pad: rows*new_cols, else the sources) is not read:
+    // such a tile (at most the last one or two) takes the exact word gather.
+    const int64_t buf_end = (PAD ? int64_t(p.out_words) : int64_t(p.in_words)) + mis;
+    g.fast = (se - g.sb) <= STAGE && se <= buf_end;
     g.bytes = g.span > 0 && g.fast ? uint32_t(se - g.sb) * 4u : 0u;
     g.base_rel = int32_t(p.src0 + g.row0 * Cw - slo);
 
@@ -143,7 +147,9 @@ __device__ __forceinline__ void wait_loaded(const uint64_t* __restrict__ status,
         const int64_t idx = base + lane;
         bool ok = idx > hi || status_current(ld_relaxed_gpu(status_ptr(status, idx)), epoch);
         uint32_t ns = 32;
+        SpinGuard guard;
         while (!__all_sync(0xffffffffu, ok)) {
+            guard.check("regular window wait");
             __nanosleep(ns);
             ns = ns < 512 ? ns * 2 : 512;
             if (!ok) ok = status_current(ld_relaxed_gpu(status_ptr(status, idx)), epoch);

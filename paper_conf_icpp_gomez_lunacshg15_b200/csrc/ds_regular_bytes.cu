@@ -88,9 +88,12 @@ __device__ void tile_geometry_b(const RegBParams& p, int64_t k, TileGeomB& g) {
     }
     g.slo = slo;
     g.span = shi >= slo ? shi - slo + 1 : 0;
-    g.sb = (slo + mis) & ~int64_t(15);
+    g.sb = (slo + mis) & ~int64_t(15);  // lead bytes: inside the 16-byte chunk holding slo
     const int64_t se = (slo + mis + g.span + 15) & ~int64_t(15);
-    g.bytes = (g.span > 0 && se - g.sb <= kBStageBytes) ? uint32_t(se - g.sb) : 0u;
+    // whole 16-byte chunks, never past the end of the caller's buffer (pad:
+    // rows*new_cols bytes, unpad: rows*cols): else the exact byte gather
+    const int64_t buf_end = (PAD ? int64_t(p.out_bytes) : int64_t(p.in_bytes)) + mis;
+    g.bytes = (g.span > 0 && se - g.sb <= kBStageBytes && se <= buf_end) ? uint32_t(se - g.sb) : 0u;
     g.base_rel = int32_t(g.row0 * Cb - slo);
 
     // Earlier-ticketed tiles whose sources lie in this tile's output bytes.
@@ -127,7 +130,9 @@ __device__ __forceinline__ void wait_loaded_b(const uint64_t* __restrict__ statu
         const int64_t idx = base + lane;
         bool ok = idx > hi || status_current(ld_relaxed_gpu(status_ptr(status, idx)), epoch);
         uint32_t ns = 32;
+        SpinGuard guard;
         while (!__all_sync(0xffffffffu, ok)) {
+            guard.check("regular window wait");
             __nanosleep(ns);
             ns = ns < 512 ? ns * 2 : 512;
             if (!ok) ok = status_current(ld_relaxed_gpu(status_ptr(status, idx)), epoch);

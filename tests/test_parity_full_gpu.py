@@ -89,3 +89,66 @@ def test_c5_compact_4g_single_gpu():
     exp = dev.cpu().numpy().view(np.uint32).copy()
     m = oracle.compact(exp, 0)
     _run(dev, exp, m, "compact", 0)
+
+
+@pytest.mark.parametrize("R,C,NC,eb", [(16384, 16383, 16384, 4), (16384, 16383, 16384, 8),
+                                       (12000, 11999, 12000, 4)])
+def test_pad_unpad_bench_shapes(R, C, NC, eb):
+    """The bench's pad / unpad rows at >= 256M elements (f32 and 8-byte
+    elements) and the Table-I shape: whole buffer."""
+    dev = dsgen.matrix_input(R, C, NC, eb, device="cuda")
+    exp = dev.cpu().numpy().view(np.uint32).copy()
+    oracle.pad(exp, R, C, NC, eb)
+    libds.ds_pad_ex(dev, R, C, NC, eb, None, None)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev.cpu().numpy().view(np.uint32), exp)
+    oracle.unpad(exp, R, NC, C, eb)
+    libds.ds_unpad_ex(dev, R, NC, C, eb, None)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev.cpu().numpy().view(np.uint32), exp)
+
+
+def test_pad_unpad_bytes_bench_shape():
+    """1-byte elements at 16384 x 16383 <-> 16384 (the byte-granular kernel)."""
+    R, C, NC = 16384, 16383, 16384
+    g = torch.Generator(device="cuda").manual_seed(7)
+    dev = torch.randint(0, 256, (R * NC,), dtype=torch.uint8, device="cuda", generator=g)
+    exp = dev.cpu().numpy().copy()
+    oracle.pad(exp, R, C, NC, 1)
+    libds.ds_pad_ex(dev, R, C, NC, 1, None, None)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev.cpu().numpy(), exp)
+    oracle.unpad(exp, R, NC, C, 1)
+    libds.ds_unpad_ex(dev, R, NC, C, 1, None)
+    torch.cuda.synchronize()
+    assert np.array_equal(dev.cpu().numpy(), exp)
+
+
+def test_partition_256m():
+    """The bench's partition row (in place through aux), whole buffer."""
+    n = 1 << 28
+    dev = dsgen.select_input(n, dsgen.seed_for(5), device="cuda")
+    t = dsgen.select_threshold(0.5) & 0xFFFFFFFF
+    exp = dev.cpu().numpy().view(np.uint32).copy()
+    m = oracle.partition(exp, oracle.PRED_I32_GT, t)
+    aux = torch.empty_like(dev)
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    libds.ds_partition_ex(dev, n, libds.DS_PRED_I32_GT, t, aux, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == m
+    assert np.array_equal(dev.cpu().numpy().view(np.uint32), exp)
+
+
+@pytest.mark.parametrize("mis", [1, 3])
+def test_c4_compact_1g_misaligned(mis):
+    """Full size at a misaligned pointer (tile grid shifted by mis words)."""
+    n = (1 << 30) - 5
+    base = dsgen.compact_input(n + 8, 0.5, dsgen.seed_for(3, 7), kind="f32", device="cuda")
+    dev = base[mis:mis + n]
+    exp = base.cpu().numpy().view(np.uint32).copy()
+    m = oracle.compact(exp[mis:mis + n], 0)
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    libds.ds_compact_ex(dev, n, 0, d_n, None)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == m
+    assert np.array_equal(base.cpu().numpy().view(np.uint32), exp)

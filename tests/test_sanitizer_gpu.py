@@ -1,0 +1,75 @@
+"""T4: compute-sanitizer over a small invocation of every kernel
+(tests/sanitize_driver.py), and failure detection: the
+DS_SPIN_CAP_NS build turns a lost tile publication into DS_ERROR_CUDA
+instead of a hang."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+from paper_conf_icpp_gomez_lunacshg15_b200 import build
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+pytestmark = pytest.mark.gpu
+
+
+def _sanitizer():
+    for cand in ("/usr/local/cuda/bin/compute-sanitizer", shutil.which("compute-sanitizer")):
+        if cand and os.path.exists(cand):
+            return cand
+    pytest.skip("compute-sanitizer not found")
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("tool,part", [("memcheck", "all"), ("synccheck", "irregular"),
+                                       ("synccheck", "regular"), ("racecheck", "regular")])
+def test_compute_sanitizer(tool, part):
+    """No memcheck error (out-of-bounds / misaligned accesses, with arrays that
+    end exactly at their cudaMalloc'd end), no synccheck hazard (barriers,
+    mbarriers), no racecheck hazard in the regular kernels' shared memory."""
+    env = dict(os.environ, PYTORCH_NO_CUDA_MEMORY_CACHING="1")
+    cmd = [_sanitizer(), "--tool", tool, "--error-exitcode", "9", "--print-limit", "20",
+           sys.executable, os.path.join(HERE, "sanitize_driver.py"), part]
+    r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=3000)
+    out = r.stdout[-6000:] + r.stderr[-6000:]
+    assert r.returncode == 0, out
+    assert "sanitize driver OK" in r.stdout, out
+
+
+def test_spin_cap_build_has_no_false_positive():
+    """Every wait loop armed with a 2 s cap: the stress driver still passes."""
+    lib = build.build("spincap")
+    env = dict(os.environ, LIBDS_PATH=lib)
+    r = subprocess.run([sys.executable, os.path.join(HERE, "stress_driver.py"), "3"],
+                       env=env, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+
+
+_HANG_PROBE = r"""
+import sys, torch
+sys.path.insert(0, {root!r})
+from paper_conf_icpp_gomez_lunacshg15_b200 import libds
+a = torch.ones(20 * 8192 + 3, dtype=torch.int32, device="cuda")
+try:
+    libds.ds_compact(a, a.numel(), 0)
+except libds.DSError as e:
+    print("DSERROR", e)
+    sys.exit(0)
+print("NO ERROR")
+sys.exit(1)
+"""
+
+
+def test_lost_tile_is_reported_not_hung():
+    """Tile 5 never publishes (DS_DEBUG_DROP_TILE): with the spin cap the
+    launch traps within ~0.2 s of waiting and the blocking call returns
+    DS_ERROR_CUDA; the process ends instead of hanging."""
+    lib = build.build("hang")
+    env = dict(os.environ, LIBDS_PATH=lib)
+    code = _HANG_PROBE.format(root=os.path.dirname(HERE))
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+    assert "DSERROR" in r.stdout and "DS_ERROR_CUDA" in r.stdout, r.stdout
+    assert "exceeded DS_SPIN_CAP_NS" in r.stdout + r.stderr

@@ -82,7 +82,10 @@ def role_samples(rep, src_file):
         return next((i + 1 for i, x in enumerate(lines) if pat in x), None)
     marks = sorted((v, k) for k, v in {
         "look-back": find("uint64_t lookback("), "look-back (local chain)": find("uint64_t lookback_window("),
-        "store helpers": find("void store_segment("), "kernel setup": find("mbar_wait_or_end("),
+        "storers (STG helper)": find("void store_segment("), "storers (re-phase)": find("void rephase("),
+        "end-aware waits": find("bool mbar_wait_or_end("),
+        "rankers (keep bits)": find("uint32_t keep_bits4("),
+        "kernel setup": find("__global__ void __launch_bounds__"),
         "producer": find("---- producer"), "rankers": find("---- ranker warps"),
         "resolvers": find("---- resolver warps"), "storers": find("---- storer warps"),
         "host": find("struct LaunchCache")}.items() if v)
