@@ -143,6 +143,14 @@ constexpr int kSeg = kT / kGroupWarps;    // contiguous words ranked by one warp
 constexpr int kRounds = kSeg / 128;       // rounds of 4 words per lane
 constexpr int kPacks = (kRounds + 3) / 4; // registers of packed 8-bit round counts
 static_assert(kRankGroups == 1 || kRankGroups == 2, "named barriers 1 and 3 serve the ranker groups");
+// Every ranker lane arrives on the tile's "ranked" barrier after its own
+// compaction stores (else lane 0 for the warp, after __syncwarp: the same
+// ordering under the PTX model, but not one compute-sanitizer racecheck models).
+#ifndef DS_IRR_ALL_LANES_ARRIVE
+#define DS_IRR_ALL_LANES_ARRIVE 1
+#endif
+constexpr bool kAllLanesArrive = DS_IRR_ALL_LANES_ARRIVE;
+constexpr int kRankedArrivals = kAllLanesArrive ? kRT : kGroupWarps;
 static_assert(kRounds % 4 == 0, "whole packs of rounds");
 constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
 constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
@@ -208,14 +216,17 @@ __device__ __forceinline__ uint32_t lds_u32(uint32_t addr) {
 __device__ __forceinline__ void sts_u32(uint32_t addr, uint32_t v) {
     asm volatile("st.shared.u32 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
 }
-// The ring's free counter: storer -> rankers, ordered at CTA scope (the
-// storer's bulk reads of the freed words completed before its release).
+// Shared-memory flags between roles (the ring's free counter, the ring
+// allocation order, the end marker), ordered at CTA scope: written with a
+// release, read with an acquire.  Both are atomics (exchange / or 0) rather
+// than st.release / ld.acquire: same ordering, and compute-sanitizer racecheck
+// models atomics but not plain release/acquire accesses.
 __device__ __forceinline__ void st_release_cta_smem(uint32_t* p, uint32_t v) {
-    asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_addr(p)), "r"(v) : "memory");
+    asm volatile("atom.release.cta.shared::cta.exch.b32 _, [%0], %1;" ::"r"(smem_addr(p)), "r"(v) : "memory");
 }
 __device__ __forceinline__ uint32_t ld_acquire_cta_smem(const uint32_t* p) {
     uint32_t v;
-    asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_addr(p)) : "memory");
+    asm volatile("atom.acquire.cta.shared::cta.or.b32 %0, [%1], 0;" : "=r"(v) : "r"(smem_addr(p)) : "memory");
     return v;
 }
 // Free input stages (bit s): released (or) by the ranker / storer that is done
@@ -361,8 +372,8 @@ __device__ __forceinline__ void store_segment(uint32_t* base, uint64_t d0, uint3
 }
 
 // a7 helper: move the cnt words seg[0, cnt) to seg[ph, ph + cnt) in shared
-// memory (ph = 1..3; seg 16-byte aligned with >= 4 readable words before it
-// and >= 6 writable words after the segment).  Destination chunk c (words
+// memory (ph = 1..3; seg 16-byte aligned with >= 6 writable words after the
+// segment).  Destination chunk c (words
 // [4c, 4c+4)) takes source words [4c-ph, 4c+4-ph): two aligned vector loads.
 // Writing chunk c destroys sources of chunk c+1 only, so the chunks go in
 // descending rounds, each reading everything before writing.
@@ -377,7 +388,10 @@ __device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph
         for (int u = 0; u < kU; ++u) {
             const int32_t c = lo + u * kSTT + st;
             if (c >= 0 && c < hi) {
-                const u32x4 a = *reinterpret_cast<const u32x4*>(seg + 4 * c - 4);
+                // chunk 0's leading words are dead (never stored): they are taken
+                // from chunk 0 itself, since the words before seg may belong to
+                // another tile's region
+                const u32x4 a = *reinterpret_cast<const u32x4*>(seg + 4 * (c > 0 ? c : 1) - 4);
                 const u32x4 b = *reinterpret_cast<const u32x4*>(seg + 4 * c);
                 switch (ph) {  // uniform
                 case 1: w[u] = u32x4{a.w, b.x, b.y, b.z}; break;
@@ -409,7 +423,7 @@ constexpr uint32_t kEndPollNs = DS_IRR_END_POLL_NS;
 #define DS_IRR_TESTWAIT 1
 #endif
 __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
-                                                 const volatile uint32_t* s_end, uint32_t k) {
+                                                 const uint32_t* s_end, uint32_t k) {
     if (DS_IRR_TESTWAIT && mbar_test_wait(bar, parity)) return true;  // no suspension if already complete
     SpinGuard guard;
     while (true) {
@@ -417,7 +431,7 @@ __device__ __forceinline__ bool mbar_wait_or_end(uint64_t* bar, uint32_t parity,
         if (mbar_try_wait(bar, parity, kEndPollNs)) return true;
         // Strictly beyond the end marker: the position holding the marker
         // itself still gets its arrival and must pass it on.
-        if (*s_end < k) return false;
+        if (ld_acquire_cta_smem(s_end) < k) return false;
     }
 }
 
@@ -459,7 +473,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         bar_ranked[kSlots], bar_resolved[kSlots], bar_stored[kSlots];
     __shared__ SlotMeta meta[kSlots];
     __shared__ uint32_t s_epoch;
-    __shared__ volatile uint32_t s_end;  // ring position of the end marker
+    __shared__ uint32_t s_end;           // ring position of the end marker (release / acquire)
     __shared__ uint32_t s_freed;         // output-ring words released by the storers (monotone)
     __shared__ uint32_t s_stages;        // free input stages (bit mask)
     __shared__ uint32_t s_alloc;         // ring positions whose ring decision is out
@@ -470,7 +484,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             mbar_init(&bar_loaded[o], 1);
             mbar_init(&bar_drawn[o], 1);
             mbar_init(&bar_counted[o], 1);
-            mbar_init(&bar_ranked[o], kGroupWarps);
+            mbar_init(&bar_ranked[o], kRankedArrivals);
             mbar_init(&bar_resolved[o], 1);
             mbar_init(&bar_stored[o], 1);
         }
@@ -504,7 +518,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             if (k == 0) s_epoch = epoch;
             if (t >= p.ntiles) {  // one failed draw per CTA ends its work
                 meta[o].tile = kNoTile;
-                s_end = k;
+                st_release_cta_smem(&s_end, k);
                 mbar_arrive(&bar_drawn[o]);
                 mbar_arrive(&bar_loaded[o]);
                 // End markers for the other resolvers' next positions, so each of
@@ -764,8 +778,12 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
                 }
                 fence_proxy_async_smem();  // the compacted words leave through a bulk store
             }
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is compacted
+            if (kAllLanesArrive) {
+                mbar_arrive(&bar_ranked[o]);  // each lane's compaction stores are released by its own arrival
+            } else {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&bar_ranked[o]);  // this warp's part of the tile is compacted
+            }
             if (rt == 0) trace_event(p.trace, t, 15, globaltimer());
         }
     } else if (warp < kWarpStorer0) {

@@ -219,7 +219,7 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
         for (int s = 0; s < kStages; ++s) {
-            mbar_init(&bar_full[s], 1);
+            mbar_init(&bar_full[s], 32);  // every producer lane arrives (its stage writes, slow path)
             mbar_init(&bar_loaded[s], 1);
             mbar_init(&bar_empty[s], kConsumerWarps);
         }
@@ -242,10 +242,9 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
             t = __shfl_sync(0xffffffffu, t, 0);
             epoch = __shfl_sync(0xffffffffu, epoch, 0);
             if (t >= p.ntiles) {  // one failed draw per CTA ends its work
-                if (lane == 0) {
-                    meta[s].g.k = kNoTile;
-                    mbar_arrive(&bar_full[s]);
-                }
+                if (lane == 0) meta[s].g.k = kNoTile;
+                __syncwarp();
+                mbar_arrive(&bar_full[s]);
                 break;
             }
             const int64_t kt = PAD ? int64_t(p.ntiles) - 1 - t : int64_t(t);
@@ -264,10 +263,13 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
             __syncwarp();
             const TileGeom& g = meta[s].g;
             if (!g.bytes) {
-                // slow path, or no sources at all (all fill): complete the full
-                // barrier's phase by a plain arrival to keep its parity in step
+                // slow path, or no sources at all (all fill): every lane arrives
+                // after its own stage writes (so each write is ordered before the
+                // phase completes, without relying on the warp barrier)
                 if (g.span > 0) gather_slow<PAD>(p, g, stage, lane);
-                if (lane == 0) mbar_arrive(&bar_full[s]);
+                mbar_arrive(&bar_full[s]);
+            } else if (lane != 0) {
+                mbar_arrive(&bar_full[s]);  // lane 0 arrived with the copy's byte count
             }
         }
     } else if (warp == 1) {

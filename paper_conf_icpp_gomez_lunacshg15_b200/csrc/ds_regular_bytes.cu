@@ -200,7 +200,7 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
         for (int s = 0; s < kBStages; ++s) {
-            mbar_init(&bar_full[s], 1);
+            mbar_init(&bar_full[s], 32);  // every producer lane arrives (its stage writes, slow path)
             mbar_init(&bar_loaded[s], 1);
             mbar_init(&bar_empty[s], kBConsumerWarps);
         }
@@ -220,10 +220,9 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
             t = __shfl_sync(0xffffffffu, t, 0);
             epoch = __shfl_sync(0xffffffffu, epoch, 0);
             if (t >= p.ntiles) {
-                if (lane == 0) {
-                    geo[s].k = kNoTileB;
-                    mbar_arrive(&bar_full[s]);
-                }
+                if (lane == 0) geo[s].k = kNoTileB;
+                __syncwarp();
+                mbar_arrive(&bar_full[s]);
                 break;
             }
             const int64_t kt = PAD ? int64_t(p.ntiles) - 1 - t : int64_t(t);
@@ -242,8 +241,11 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
             __syncwarp();
             const TileGeomB& g = geo[s];
             if (!g.bytes) {
+                // every lane arrives after its own stage writes
                 if (g.span > 0) gather_slow_b<PAD>(p, g, stage, lane);
-                if (lane == 0) mbar_arrive(&bar_full[s]);
+                mbar_arrive(&bar_full[s]);
+            } else if (lane != 0) {
+                mbar_arrive(&bar_full[s]);  // lane 0 arrived with the copy's byte count
             }
         }
     } else if (warp == 1) {

@@ -24,7 +24,8 @@ def _sanitizer():
 
 @pytest.mark.slow
 @pytest.mark.parametrize("tool,part", [("memcheck", "all"), ("synccheck", "irregular"),
-                                       ("synccheck", "regular"), ("racecheck", "regular")])
+                                       ("synccheck", "regular"), ("racecheck", "regular"),
+                                       ("racecheck", "irregular")])
 def test_compute_sanitizer(tool, part):
     """No memcheck error (out-of-bounds / misaligned accesses, with arrays that
     end exactly at their cudaMalloc'd end), no synccheck hazard (barriers,
