@@ -143,5 +143,34 @@ def _more(rep, d_n):
         assert np.array_equal(u32(a), exp), ("slide", rep, shift)
 
 
+def main_large(reps):
+    """Full-size reordering stress (R10): 256M-word compaction at f = 0.1 /
+    0.5 / 0.9 and unique, `reps` launches each, every result compared with
+    the oracle's (computed once per input)."""
+    n = 1 << 28
+    cases = []
+    for f in (0.1, 0.5, 0.9):
+        cases.append(("compact", dsgen.compact_input(n, f, 4000 + int(10 * f), device="cuda")))
+    cases.append(("unique", dsgen.unique_runs_input(n, 0.4, 4100, device="cuda")))
+    d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    for kind, src in cases:
+        exp = u32(src)
+        m = oracle.unique(exp) if kind == "unique" else oracle.compact(exp, 0)
+        want = torch.from_numpy(exp.view(np.int32)).cuda()
+        work = torch.empty_like(src)
+        for rep in range(reps):
+            work.copy_(src)
+            if kind == "unique":
+                libds.ds_unique_ex(work, n, None, 0, d_n, None)
+            else:
+                libds.ds_compact_ex(work, n, 0, d_n, None)
+            assert int(d_n.item()) == m and torch.equal(work, want), (kind, rep)
+        del want, work
+    print(f"stress OK: large, {reps} reps x {len(cases)} inputs with {libds.LIB_PATH}")
+
+
 if __name__ == "__main__":
-    main(int(sys.argv[1]) if len(sys.argv) > 1 else 10)
+    if len(sys.argv) > 2 and sys.argv[2] == "large":
+        main_large(int(sys.argv[1]))
+    else:
+        main(int(sys.argv[1]) if len(sys.argv) > 1 else 10)

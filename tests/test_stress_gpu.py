@@ -21,3 +21,18 @@ def test_delay_injection_parity(variant):
                        env=env, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     assert "stress OK" in r.stdout
+
+
+@pytest.mark.gpu
+@pytest.mark.slow
+@pytest.mark.parametrize("variant", ["stress", "strict", "release"])
+def test_relaxed_ordering_full_size(variant):
+    """The relaxed status ordering (R10) at full size: 50 launches each of
+    256M-word compaction at f = 0.1 / 0.5 / 0.9 and unique, with random
+    per-CTA delays (stress) and in the release build, all bit-exact."""
+    lib = build.build(variant)
+    env = dict(os.environ, LIBDS_PATH=lib)
+    r = subprocess.run([sys.executable, os.path.join(HERE, "stress_driver.py"), "50", "large"],
+                       env=env, capture_output=True, text=True, timeout=1800)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    assert "stress OK: large" in r.stdout
