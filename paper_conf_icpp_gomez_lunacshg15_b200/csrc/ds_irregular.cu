@@ -37,6 +37,8 @@
 // tiles; a drawn tile reaches AGG without waiting on any other tile; a ranker
 // waiting for ring space waits only for this CTA's lower tiles, whose
 // aggregates (and so all their predecessors' statuses) are already out.
+#include <type_traits>
+
 #include "ds_device.cuh"
 #include "ds_internal.h"
 
@@ -599,62 +601,71 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             uint32_t kb = 0, P[kPacks];
 #pragma unroll
             for (int i = 0; i < kPacks; ++i) P[i] = 0;
-            // unique: rot[r] = lane l-1's last word of round r; lane 0 receives lane 31's,
-            // which is lane 0's predecessor in round r+1 (one shuffle per round)
-            uint32_t rot_z = 0, rot_w = 0;
+            // Keep bits of all rounds.  Only tile 0 (the array's first word, lead
+            // words before ptr) and the last tile need range checks: the guarded
+            // variant is a separate, compile-time copy, so every other tile runs
+            // the pass without a per-round branch.
+            auto keep_pass = [&](auto guard_tag) {
+                constexpr bool G = decltype(guard_tag)::value;
+                // unique: lane l-1's last word of round r; lane 0 receives lane 31's,
+                // which is lane 0's predecessor in round r+1 (one shuffle per round)
+                uint32_t rot_z = 0, rot_w = 0;
 #pragma unroll
-            for (int r = 0; r < kRounds; ++r) {
-                const uint32_t x0 = uint32_t(xs + 128 * r + 4 * lane);
-                uint32_t b;
-                if constexpr (Op::kWide) {
-                    uint32_t pz = 0, pw = 0;
-                    if constexpr (Op::kUnique) {
-                        // element before (x, y): lane l-1's (z, w), lane 31 of the previous
-                        // round, or the two staged words before the segment
-                        const uint32_t tz = __shfl_sync(kFull, v[r].z, (lane + 31) & 31);
-                        const uint32_t tw = __shfl_sync(kFull, v[r].w, (lane + 31) & 31);
-                        if (lane != 0) {
-                            pz = tz, pw = tw;
-                        } else if (r > 0) {
-                            pz = rot_z, pw = rot_w;
-                        } else {
-                            pz = lds_u32(st_b + 4u * uint32_t(xs - 2));
-                            pw = lds_u32(st_b + 4u * uint32_t(xs - 1));
+                for (int r = 0; r < kRounds; ++r) {
+                    const uint32_t x0 = uint32_t(xs + 128 * r + 4 * lane);
+                    uint32_t b;
+                    if constexpr (Op::kWide) {
+                        uint32_t pz = 0, pw = 0;
+                        if constexpr (Op::kUnique) {
+                            // element before (x, y): lane l-1's (z, w), lane 31 of the previous
+                            // round, or the two staged words before the segment
+                            const uint32_t tz = __shfl_sync(kFull, v[r].z, (lane + 31) & 31);
+                            const uint32_t tw = __shfl_sync(kFull, v[r].w, (lane + 31) & 31);
+                            if (lane != 0) {
+                                pz = tz, pw = tw;
+                            } else if (r > 0) {
+                                pz = rot_z, pw = rot_w;
+                            } else {
+                                pz = lds_u32(st_b + 4u * uint32_t(xs - 2));
+                                pw = lds_u32(st_b + 4u * uint32_t(xs - 1));
+                            }
+                            rot_z = tz, rot_w = tw;
                         }
-                        rot_z = tz, rot_w = tw;
+                        b = keep_bits4_wide<Op>(v[r], pz, pw, uint64_t(p.value_hi) << 32 | p.value);
+                        if (Op::kUnique && G && t == 0) {  // the array's first element is kept
+                            if (x0 == xlo) b |= 3u;
+                            if (x0 + 2 == xlo) b |= 12u;
+                        }
+                    } else {
+                        uint32_t pw = 0;
+                        if constexpr (Op::kUnique) {
+                            // word before x0: lane l-1's last word, lane 31 of the previous
+                            // round, or the staged word before the segment (P:280 for xs = 0)
+                            const uint32_t tw = __shfl_sync(kFull, v[r].w, (lane + 31) & 31);
+                            pw = lane != 0 ? tw : r > 0 ? rot_w : lds_u32(st_b + 4u * uint32_t(xs - 1));
+                            rot_w = tw;
+                        }
+                        b = keep_bits4<Op>(v[r], pw, p.value);
+                        if (Op::kUnique && G && t == 0 && x0 <= xlo && xlo < x0 + 4) {
+                            // the array's first word (R18): kept unless it equals the halo word
+                            const uint32_t j = xlo - x0;
+                            const uint32_t w0 = j == 0 ? v[r].x : j == 1 ? v[r].y : j == 2 ? v[r].z : v[r].w;
+                            const bool k0 = !has_hprev || w0 != hprev;
+                            b = (b & ~(1u << j)) | (uint32_t(k0) << j);
+                        }
                     }
-                    b = keep_bits4_wide<Op>(v[r], pz, pw, uint64_t(p.value_hi) << 32 | p.value);
-                    if (Op::kUnique && guarded && t == 0) {  // the array's first element is kept
-                        if (x0 == xlo) b |= 3u;
-                        if (x0 + 2 == xlo) b |= 12u;
+                    if (G) {
+                        // words outside [xlo, xhi) are not elements of the array
+                        const uint32_t lo_ok = x0 >= xlo ? 15u : (15u << (xlo - x0)) & 15u;
+                        const uint32_t hi_ok = x0 + 4 <= xhi ? 15u : x0 >= xhi ? 0u : (1u << (xhi - x0)) - 1u;
+                        b &= lo_ok & hi_ok;
                     }
-                } else {
-                    uint32_t pw = 0;
-                    if constexpr (Op::kUnique) {
-                        // word before x0: lane l-1's last word, lane 31 of the previous
-                        // round, or the staged word before the segment (P:280 for xs = 0)
-                        const uint32_t tw = __shfl_sync(kFull, v[r].w, (lane + 31) & 31);
-                        pw = lane != 0 ? tw : r > 0 ? rot_w : lds_u32(st_b + 4u * uint32_t(xs - 1));
-                        rot_w = tw;
-                    }
-                    b = keep_bits4<Op>(v[r], pw, p.value);
-                    if (Op::kUnique && guarded && t == 0 && x0 <= xlo && xlo < x0 + 4) {
-                        // the array's first word (R18): kept unless it equals the halo word
-                        const uint32_t j = xlo - x0;
-                        const uint32_t w0 = j == 0 ? v[r].x : j == 1 ? v[r].y : j == 2 ? v[r].z : v[r].w;
-                        const bool k0 = !has_hprev || w0 != hprev;
-                        b = (b & ~(1u << j)) | (uint32_t(k0) << j);
-                    }
+                    kb |= b << (4 * r);
+                    P[r / 4] += uint32_t(__popc(b)) << (8 * (r % 4));
                 }
-                if (guarded) {
-                    // words outside [xlo, xhi) are not elements of the array
-                    const uint32_t lo_ok = x0 >= xlo ? 15u : (15u << (xlo - x0)) & 15u;
-                    const uint32_t hi_ok = x0 + 4 <= xhi ? 15u : x0 >= xhi ? 0u : (1u << (xhi - x0)) - 1u;
-                    b &= lo_ok & hi_ok;
-                }
-                kb |= b << (4 * r);
-                P[r / 4] += uint32_t(__popc(b)) << (8 * (r % 4));
-            }
+            };
+            if (guarded) keep_pass(std::true_type{});
+            else keep_pass(std::false_type{});
             // exclusive offsets of every lane in all rounds (8-bit fields, <= 128 each)
             uint32_t inc[kPacks];
 #pragma unroll
