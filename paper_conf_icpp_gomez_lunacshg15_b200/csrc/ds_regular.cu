@@ -167,9 +167,13 @@ __device__ __forceinline__ void wait_loaded(const uint64_t* __restrict__ status,
 #endif
 constexpr int kConsumerWarps = DS_REG_CONSUMER_WARPS;
 constexpr int kCT = 32 * kConsumerWarps;  // consumer threads
-constexpr int kItems = 8192 / kCT;        // output words per consumer thread
+#ifndef DS_REG_TILE
+#define DS_REG_TILE 8192
+#endif
+constexpr int kItems = DS_REG_TILE / kCT; // output words per consumer thread
 constexpr int kVec = kItems / 4;
-constexpr int kT = kCT * kItems;          // 8192 output words = 32 KB per tile
+constexpr int kT = kCT * kItems;          // output words per tile (8192 = 32 KB)
+static_assert(kItems % 4 == 0, "whole 128-bit vectors per consumer thread");
 constexpr int kStageWords = kT + 512;     // staged source span cap (words)
 constexpr int kStages = DS_REG_STAGES;
 constexpr int kThreads = 32 * (2 + kConsumerWarps);  // producer, publisher, consumers
