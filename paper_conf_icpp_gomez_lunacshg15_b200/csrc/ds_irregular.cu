@@ -140,7 +140,10 @@ constexpr int kRankWarps = 16;
 constexpr int kRankGroups = DS_IRR_RANK_GROUPS;   // ranker groups, each on its own tile
 constexpr int kGroupWarps = kRankWarps / kRankGroups;
 constexpr int kRT = 32 * kGroupWarps;     // threads of one ranker group
-constexpr int kT = 8192;                  // words per tile (32 KB)
+#ifndef DS_IRR_TILE
+#define DS_IRR_TILE 8192
+#endif
+constexpr int kT = DS_IRR_TILE;           // words per tile (8192 = 32 KB)
 constexpr int kSeg = kT / kGroupWarps;    // contiguous words ranked by one warp
 constexpr int kRounds = kSeg / 128;       // rounds of 4 words per lane
 constexpr int kPacks = (kRounds + 3) / 4; // registers of packed 8-bit round counts
@@ -173,7 +176,7 @@ constexpr int kStageWords = kT + kPre + 32;
 // ring (the stage is free as soon as every ranker holds its words in
 // registers); the storers drain the ring in tile order once the prefix is
 // known.  Everything left of the 227 KB after the input stages.
-constexpr int kStaticSmem = 2560;  // barriers, slot metadata (static shared memory; ptxas reports 2176 B)
+constexpr int kStaticSmem = 128 * kSlots + 512;  // barriers + slot metadata (static shared memory; ptxas: 2048 B at 16 slots)
 #ifndef DS_IRR_RING_WORDS
 #define DS_IRR_RING_WORDS (((227 * 1024 - kStaticSmem - 128) / 4 - kInStages * kStageWords) / 32 * 32)
 #endif
@@ -508,6 +511,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             // once, one compacted in place only once stored)
             uint32_t m;
             SpinGuard guard;
+            const uint64_t t_claim = p.trace ? globaltimer() : 0;  // diagnostics: stage wait
             while ((m = ld_acquire_cta_smem(&s_stages)) == 0u) {
                 guard.check("irregular producer stage wait");
                 __nanosleep(32);
@@ -538,6 +542,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             mbar_arrive(&bar_drawn[o]);  // the resolver starts this tile's look-back now
             trace_event(p.trace, t, 0, globaltimer());
             trace_event(p.trace, t, 7, smid());
+            trace_event(p.trace, t, 13, t_claim);  // start of the wait for a free input stage
             debug_delay(t, 0);
             const uint64_t tb = uint64_t(t) * kT;
             const uint64_t end = tb + kT < p.hi ? tb + kT : p.hi;
@@ -693,7 +698,6 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             if (lane == 0) meta[o].wtot[rw] = wrun;
             if (rt == 0) {
                 meta[o].freed_snap = ld_acquire_cta_smem(&s_freed);  // one ring view for the group
-                trace_event(p.trace, t, 13, globaltimer());
             }
             named_bar_sync(gbar, kRT);  // warp totals written; every ranker holds its words
             if (rt == 0) trace_event(p.trace, t, 14, globaltimer());
@@ -752,6 +756,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint32_t rpos = hp;
             if (rt == 0) {
                 meta[o].ring_pos = in_ring ? rpos : kNoTile;
+                trace_event(p.trace, t, 7, smid() | uint64_t(in_ring) << 16);  // diagnostics: ring or in place
                 meta[o].ring_end = in_ring ? h + need : h0;
                 meta[o].ring_hpos = in_ring ? hp + need : hp0;
                 if (kRankGroups > 1) st_release_cta_smem(&s_alloc, k + 1);
