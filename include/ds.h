@@ -263,8 +263,8 @@ int ds_version(void);
 
 /* Tile size of a kernel family, for tests that aim at tile edges: the
  * irregular kernel's input tile and the regular kernel's output tile in
- * 4-byte words, the byte-granular regular kernel's output tile in bytes
- * (0 for an unknown id).  Tiles start at the 16-byte boundary at or below
+ * 4-byte words, the byte-granular regular kernel's output tile in bytes for
+ * outputs of 64 MiB or more (16384 bytes below; 0 for an unknown id).  Tiles start at the 16-byte boundary at or below
  * ptr, so tile k covers words [16B-aligned base + kT, ...).              */
 typedef enum ds_kernel {
     DS_KERNEL_IRREGULAR = 0,      /* compact / select / unique / partition */

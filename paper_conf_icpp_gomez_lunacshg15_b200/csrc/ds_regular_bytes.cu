@@ -28,14 +28,27 @@ constexpr int64_t kNoTileB = -1;
 #endif
 constexpr int kBConsumerWarps = DS_REGB_CONSUMER_WARPS;
 constexpr int kBCT = 32 * kBConsumerWarps;
-constexpr int kBChunks = 2048 / kBCT;         // 16-byte chunks per consumer thread
-constexpr int kTB = kBCT * kBChunks * 16;     // 32768 output bytes per tile
-constexpr int kBStageBytes = kTB + 2048;      // staged source span cap
-constexpr int kBStageAlloc = kBStageBytes + 32;  // vector reads may pass the span by 16 bytes
-constexpr int kBStages = 3;
+// Output tile size TB (bytes) is a template parameter: 32 KB tiles for large
+// matrices; 16 KB tiles when the output is small (< kSmallOut), where 32 KB
+// tiles leave too few tiles per CTA to fill the pipeline (1-byte pad at the C2
+// shape 19.5 -> 15.4 us; at 16384 x 16384 16 KB tiles cost 15 %).
+constexpr int kTBLarge = 32768, kTBSmall = 16384;
+constexpr uint64_t kSmallOut = 64ull << 20;
+template <int TB>
+struct BCfg {
+    static constexpr int Chunks = TB / 16 / kBCT;      // 16-byte chunks per consumer thread
+    static constexpr int StageBytes = TB + 2048;       // staged source span cap
+    static constexpr int StageAlloc = StageBytes + 32; // vector reads may pass the span by 16 bytes
+    static_assert(Chunks >= 1 && Chunks * 16 * kBCT == TB, "tile size");
+    static_assert(StageBytes % 16 == 0 && StageAlloc % 16 == 0, "stage alignment");
+};
+#ifndef DS_REGB_STAGES
+#define DS_REGB_STAGES 3
+#endif
+constexpr int kBStages = DS_REGB_STAGES;
 constexpr int kBThreads = 32 * (2 + kBConsumerWarps);
-constexpr size_t kBSmem = size_t(kBStages) * kBStageAlloc;
-static_assert(kBStageBytes % 16 == 0 && kBStageAlloc % 16 == 0, "stage alignment");
+template <int TB>
+constexpr size_t smem_b() { return size_t(kBStages) * BCfg<TB>::StageAlloc; }
 
 struct RegBParams {
     uint8_t* abase;        // 16-byte-aligned base; virtual byte 0
@@ -66,8 +79,9 @@ struct TileGeomB {
 };
 
 // Closed-form geometry, the word kernel's formulas in bytes.
-template <bool PAD>
+template <bool PAD, int TB>
 __device__ void tile_geometry_b(const RegBParams& p, int64_t k, TileGeomB& g) {
+    constexpr int64_t kTB = TB;
     const int64_t Cb = p.Cb, NCb = p.NCb, mis = int64_t(p.mis);
     const int64_t V0 = k * kTB;
     g.k = k;
@@ -93,7 +107,7 @@ __device__ void tile_geometry_b(const RegBParams& p, int64_t k, TileGeomB& g) {
     // whole 16-byte chunks, never past the end of the caller's buffer (pad:
     // rows*new_cols bytes, unpad: rows*cols): else the exact byte gather
     const int64_t buf_end = (PAD ? int64_t(p.out_bytes) : int64_t(p.in_bytes)) + mis;
-    g.bytes = (g.span > 0 && se - g.sb <= kBStageBytes && se <= buf_end) ? uint32_t(se - g.sb) : 0u;
+    g.bytes = (g.span > 0 && se - g.sb <= BCfg<TB>::StageBytes && se <= buf_end) ? uint32_t(se - g.sb) : 0u;
     g.base_rel = int32_t(g.row0 * Cb - slo);
 
     // Earlier-ticketed tiles whose sources lie in this tile's output bytes.
@@ -190,8 +204,11 @@ __device__ void gather_slow_b(const RegBParams& p, const TileGeomB& g, uint8_t* 
     __syncwarp();
 }
 
-template <bool PAD>
+template <bool PAD, int TB>
 __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBParams p) {
+    constexpr int64_t kTB = TB;
+    constexpr int kBChunks = BCfg<TB>::Chunks;
+    constexpr int kBStageAlloc = BCfg<TB>::StageAlloc;
     extern __shared__ __align__(128) uint8_t smem8[];
     __shared__ __align__(8) uint64_t bar_full[kBStages], bar_loaded[kBStages], bar_empty[kBStages];
     __shared__ TileGeomB geo[kBStages];
@@ -230,7 +247,7 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
                 debug_delay(uint64_t(kt), 0);
                 trace_event(p.trace, uint64_t(kt), 0, globaltimer());
                 trace_event(p.trace, uint64_t(kt), 7, smid());
-                tile_geometry_b<PAD>(p, kt, geo[s]);
+                tile_geometry_b<PAD, TB>(p, kt, geo[s]);
                 geo_epoch[s] = epoch;
                 if (geo[s].bytes) {
                     fence_proxy_async_smem();
@@ -386,10 +403,11 @@ struct LaunchCacheB {
     int dev = -1, sms = 0, per_sm = 0;
 };
 
-template <bool PAD>
+template <bool PAD, int TB>
 cudaError_t launch_dir_b(RegBParams p, cudaStream_t s) {
+    constexpr size_t kBSmem = smem_b<TB>();
     static thread_local LaunchCacheB lc;
-    auto kern = regular_bytes_kernel<PAD>;
+    auto kern = regular_bytes_kernel<PAD, TB>;
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e != cudaSuccess) return e;
@@ -414,11 +432,17 @@ cudaError_t launch_dir_b(RegBParams p, cudaStream_t s) {
 
 }  // namespace
 
-size_t regular_bytes_tile_bytes() { return kTB; }
+size_t regular_bytes_tile_bytes() { return kTBLarge; }
+
+// Output tile bytes a launch uses.
+static int64_t tile_bytes_for(const RegBytesArgs& a) {
+    return a.rows * a.new_cols_b < kSmallOut ? kTBSmall : kTBLarge;
+}
 
 size_t regular_bytes_tiles(const RegBytesArgs& a) {
     const uint64_t mis = reinterpret_cast<uintptr_t>(a.ptr) & 15u;
-    return size_t((a.rows * a.new_cols_b + mis + kTB - 1) / kTB);
+    const int64_t tb = tile_bytes_for(a);
+    return size_t((a.rows * a.new_cols_b + mis + tb - 1) / tb);
 }
 
 cudaError_t launch_regular_bytes(const RegBytesArgs& a, Workspace& ws, cudaStream_t s) {
@@ -441,7 +465,9 @@ cudaError_t launch_regular_bytes(const RegBytesArgs& a, Workspace& ws, cudaStrea
     p.status = ws.status;
     p.ctrl = ws.ctrl;
     count_launch();
-    return a.pad ? launch_dir_b<true>(p, s) : launch_dir_b<false>(p, s);
+    if (tile_bytes_for(a) == kTBSmall)
+        return a.pad ? launch_dir_b<true, kTBSmall>(p, s) : launch_dir_b<false, kTBSmall>(p, s);
+    return a.pad ? launch_dir_b<true, kTBLarge>(p, s) : launch_dir_b<false, kTBLarge>(p, s);
 }
 
 }  // namespace ds

@@ -90,6 +90,15 @@ def run(spec):
         else:
             timeit(f"unpad {R}x{NC}->{C} eb={eb}", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, eb, None),
                    lambda m: eb * (2 * R * C), reps=30)
+    elif op in ("padbig1", "unpadbig1"):  # >= 256M 1-byte elements (byte-granular kernel)
+        R, C, NC = 16384, 16383, 16384
+        a = torch.randint(0, 256, (R * NC,), dtype=torch.uint8, device=dev)
+        if op == "padbig1":
+            timeit(f"pad {R}x{C}->{NC} eb=1", a, lambda w, d: libds.ds_pad_ex(w, R, C, NC, 1, None, None),
+                   lambda m: R * C + R * NC)
+        else:
+            timeit(f"unpad {R}x{NC}->{C} eb=1", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, 1, None),
+                   lambda m: 2 * R * C)
     elif op == "pad12k":
         R, C, NC = 12000, 11999, 12000
         a = dsgen.matrix_input(R, C, NC, 4, device=dev)
