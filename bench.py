@@ -412,7 +412,7 @@ def run_libds(args):
     flush_buf = torch.empty(1 << 27, dtype=torch.int32, device=dev)  # 512 MiB > 126 MB L2
     flush = lambda: flush_buf.sum()  # noqa: E731  (read-only flush: leaves no dirty lines)
     stream = torch.cuda.current_stream()
-    ds = ShardedDS(device=dev)
+    ds = ShardedDS(device=dev, count_exchange=args.count_exchange)
 
     def barrier():
         if world > 1:
@@ -422,9 +422,15 @@ def run_libds(args):
     def step_once(kernel_ev):
         a, b, c = kernel_ev
         a.record(stream)
-        libds.ds_compact_ex(work, n, 0, ds.d_count, stream)
-        b.record(stream)
-        ds._finish(stream)
+        if args.count_exchange == "board":
+            # the DS kernel also stores its count into every rank's count board
+            ds.local.compact_pub(work, 0, ds.d_count, ds._pub(), stream)
+            b.record(stream)
+            ds._finish_board(stream)
+        else:
+            libds.ds_compact_ex(work, n, 0, ds.d_count, stream)
+            b.record(stream)
+            ds._finish(stream)
         c.record(stream)
 
     def one_step(timed_events):
@@ -594,7 +600,10 @@ def run_libds(args):
                        "l2": "inputs 16/N GiB per rank >> 126 MB L2; L2 also flushed by reading 512 MiB "
                              "between steps",
                        "restore": "pristine shard restored by a D2D copy between steps, outside the events",
-                       "step": "ds_compact_ex + NCCL all-gather of counts + ds_shard_offsets"},
+                       "step": ("ds_compact_pub_ex (count stored into every rank's count board over peer "
+                                "memory) + ds_shard_offsets_board" if args.count_exchange == "board" else
+                                "ds_compact_ex + NCCL all-gather of counts + ds_shard_offsets"),
+                       "count_exchange": args.count_exchange},
             "frac_of_peak": round(value / world / peak, 4),
             "frac_of_nominal": round(value / world / NOMINAL_HBM_GBS, 4),
             "elems_per_s": round(N_TOTAL / (ms_per_step * 1e-3), 1),
@@ -621,6 +630,7 @@ def run_libds(args):
         if rows:
             line["rows"] = rows
         print(json.dumps(line), flush=True)
+    ds.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
@@ -638,6 +648,8 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--e2e-chunks", type=int, default=32)
     ap.add_argument("--rebalance", action="store_true", help="also time ShardedDS.rebalance (8(f)-1)")
+    ap.add_argument("--count-exchange", default="collective", choices=["collective", "board"],
+                    help="counts by NCCL all-gather (default) or through the count boards (peer memory)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "libds" and not os.environ.get("DS_BENCH_ALLOW_SHORT"):
         args.warmup = 3

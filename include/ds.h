@@ -238,6 +238,40 @@ ds_status ds_halo_entry(const void* ptr, size_t n, uint64_t* d_entry,
 ds_status ds_shard_offsets(const uint64_t* d_counts, size_t world, size_t rank,
                            uint64_t* d_result, ds_stream_t stream);
 
+/* Count boards: the fused alternative to the NCCL all-gather of the counts
+ * (DESIGN.md section 5).  Every rank owns a board of 2*world 64-bit words in
+ * its GPU's memory; every rank maps every other rank's board (CUDA IPC; peer
+ * memory over NVLink between GPUs).  The DS kernel of a shard writes its kept
+ * count, tagged with the call's `tag`, into slot 2*rank + tag%2 of EVERY
+ * board directly from its final tile (a release store per rank, no extra
+ * launch); ds_shard_offsets_board waits on the local board until every rank's
+ * word carries the tag.  A rank may run at most one call ahead of another
+ * (the two slots); tags must increase by one per call, starting at 1, and
+ * the words hold {tag:28 | count:36}.                                      */
+#define DS_IPC_HANDLE_BYTES 64
+typedef struct ds_publish {
+    uint64_t* const* d_boards; /* DEVICE array of `world` board pointers    */
+    size_t world;
+    size_t rank;
+    uint64_t tag;
+} ds_publish;
+ds_status ds_board_alloc(size_t world, uint64_t** d_board);   /* zeroed      */
+ds_status ds_board_free(uint64_t* d_board);
+ds_status ds_board_ipc_handle(const uint64_t* d_board, void* handle /* DS_IPC_HANDLE_BYTES */);
+ds_status ds_board_ipc_open(const void* handle, uint64_t** d_peer_board);
+ds_status ds_board_ipc_close(uint64_t* d_peer_board);
+/* The _ex calls plus the publication of the count (pub: HOST pointer).    */
+ds_status ds_compact_pub_ex(void* ptr, size_t n, uint32_t remove_value, uint64_t* d_out_n,
+                            const ds_publish* pub, ds_stream_t stream);
+ds_status ds_select_pub_ex(void* ptr, size_t n, int predicate_id, uint32_t param,
+                           uint64_t* d_out_n, const ds_publish* pub, ds_stream_t stream);
+ds_status ds_unique_pub_ex(void* ptr, size_t n, const uint64_t* d_halo, size_t halo_len,
+                           uint64_t* d_out_n, const ds_publish* pub, ds_stream_t stream);
+/* d_result as ds_shard_offsets; d_counts (DEVICE, may be NULL) receives all
+ * ranks' counts.                                                          */
+ds_status ds_shard_offsets_board(const uint64_t* d_board, size_t world, size_t rank, uint64_t tag,
+                                 uint64_t* d_counts, uint64_t* d_result, ds_stream_t stream);
+
 /* ---------------------------------------------------------------------
  * Utilities
  * ------------------------------------------------------------------- */

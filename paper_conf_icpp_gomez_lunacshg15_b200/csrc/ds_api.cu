@@ -158,9 +158,26 @@ ds_status irregular_ex(ds::IrregArgs a, cudaStream_t s) {
             cudaError_t e = cudaMemsetAsync(a.d_out_n, 0, sizeof(uint64_t), s);
             if (e != cudaSuccess) return fail(e, "cudaMemsetAsync");
         }
+        if (a.pub_boards) {  // an empty shard still publishes its count
+            cudaError_t e = ds::launch_publish_zero(a.pub_boards, a.pub_world, a.pub_rank, a.pub_tag, s);
+            if (e != cudaSuccess) return fail(e, "publish launch");
+        }
         return DS_SUCCESS;
     }
     return run_irregular(a, s);
+}
+
+// Peer publication of a shard's count (count boards).
+ds_status apply_publish(const ds_publish* pub, ds::IrregArgs* a) {
+    if (!pub) return DS_ERROR_INVALID_VALUE;
+    if (!pub->d_boards || pub->world == 0 || pub->world > 1024 || pub->rank >= pub->world)
+        return DS_ERROR_INVALID_VALUE;
+    if (misaligned(pub->d_boards, 8)) return DS_ERROR_INVALID_VALUE;
+    a->pub_boards = pub->d_boards;
+    a->pub_world = uint32_t(pub->world);
+    a->pub_rank = uint32_t(pub->rank);
+    a->pub_tag = pub->tag;
+    return DS_SUCCESS;
 }
 
 // Blocking form: legacy default stream, count read back through the
@@ -514,6 +531,92 @@ ds_status ds_partition(void* ptr, size_t n, int predicate_id, void* aux, size_t*
         return st;
     }
     return read_count(slot, out_n_true);
+}
+
+ds_status ds_compact_pub_ex(void* ptr, size_t n, uint32_t remove_value, uint64_t* d_out_n,
+                            const ds_publish* pub, ds_stream_t stream) {
+    ds_status st = check_irregular(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Compact, 0, remove_value, nullptr, 0, d_out_n};
+    if ((st = apply_publish(pub, &a)) != DS_SUCCESS) return st;
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_select_pub_ex(void* ptr, size_t n, int predicate_id, uint32_t param, uint64_t* d_out_n,
+                           const ds_publish* pub, ds_stream_t stream) {
+    if (predicate_id < 0 || predicate_id >= DS_PRED_COUNT) return DS_ERROR_INVALID_VALUE;
+    ds_status st = check_irregular(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Select, predicate_id, param, nullptr, 0, d_out_n};
+    if ((st = apply_publish(pub, &a)) != DS_SUCCESS) return st;
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_unique_pub_ex(void* ptr, size_t n, const uint64_t* d_halo, size_t halo_len, uint64_t* d_out_n,
+                           const ds_publish* pub, ds_stream_t stream) {
+    if (halo_len > 0 && d_halo == nullptr) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(d_halo, 8)) return DS_ERROR_INVALID_VALUE;
+    if (halo_len > 0xFFFFFFFFull) return DS_ERROR_UNSUPPORTED;
+    ds_status st = check_irregular(ptr, n, d_out_n);
+    if (st != DS_SUCCESS) return st;
+    ds::IrregArgs a{static_cast<uint32_t*>(ptr), n, ds::IrregOp::Unique, 0, 0u, d_halo, halo_len, d_out_n};
+    if ((st = apply_publish(pub, &a)) != DS_SUCCESS) return st;
+    return irregular_ex(a, reinterpret_cast<cudaStream_t>(stream));
+}
+
+ds_status ds_board_alloc(size_t world, uint64_t** d_board) {
+    if (!d_board || world == 0 || world > 1024) return DS_ERROR_INVALID_VALUE;
+    uint64_t* b = nullptr;
+    cudaError_t e = cudaMalloc(&b, 2 * world * sizeof(uint64_t));
+    if (e != cudaSuccess) return e == cudaErrorMemoryAllocation ? DS_ERROR_OUT_OF_MEMORY : fail(e, "cudaMalloc");
+    if ((e = cudaMemset(b, 0, 2 * world * sizeof(uint64_t))) != cudaSuccess) {
+        cudaFree(b);
+        return fail(e, "cudaMemset");
+    }
+    *d_board = b;
+    return DS_SUCCESS;
+}
+
+ds_status ds_board_free(uint64_t* d_board) {
+    if (!d_board) return DS_SUCCESS;
+    cudaError_t e = cudaFree(d_board);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "cudaFree");
+}
+
+ds_status ds_board_ipc_handle(const uint64_t* d_board, void* handle) {
+    if (!d_board || !handle) return DS_ERROR_INVALID_VALUE;
+    cudaIpcMemHandle_t h;
+    cudaError_t e = cudaIpcGetMemHandle(&h, const_cast<uint64_t*>(d_board));
+    if (e != cudaSuccess) return fail(e, "cudaIpcGetMemHandle");
+    static_assert(sizeof(h) == DS_IPC_HANDLE_BYTES, "IPC handle size");
+    std::memcpy(handle, &h, sizeof(h));
+    return DS_SUCCESS;
+}
+
+ds_status ds_board_ipc_open(const void* handle, uint64_t** d_peer_board) {
+    if (!handle || !d_peer_board) return DS_ERROR_INVALID_VALUE;
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle, sizeof(h));
+    void* ptr = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return fail(e, "cudaIpcOpenMemHandle");
+    *d_peer_board = static_cast<uint64_t*>(ptr);
+    return DS_SUCCESS;
+}
+
+ds_status ds_board_ipc_close(uint64_t* d_peer_board) {
+    if (!d_peer_board) return DS_ERROR_INVALID_VALUE;
+    cudaError_t e = cudaIpcCloseMemHandle(d_peer_board);
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "cudaIpcCloseMemHandle");
+}
+
+ds_status ds_shard_offsets_board(const uint64_t* d_board, size_t world, size_t rank, uint64_t tag,
+                                 uint64_t* d_counts, uint64_t* d_result, ds_stream_t stream) {
+    if (!d_board || !d_result || world == 0 || world > 1024 || rank >= world) return DS_ERROR_INVALID_VALUE;
+    if (misaligned(d_board, 8) || misaligned(d_result, 8) || misaligned(d_counts, 8)) return DS_ERROR_INVALID_VALUE;
+    cudaError_t e = ds::launch_board_offsets(d_board, world, rank, tag, d_counts, d_result,
+                                             reinterpret_cast<cudaStream_t>(stream));
+    return e == cudaSuccess ? DS_SUCCESS : fail(e, "board offsets launch");
 }
 
 ds_status ds_halo_entry(const void* ptr, size_t n, uint64_t* d_entry, ds_stream_t stream) {

@@ -32,7 +32,20 @@ struct IrregArgs {
     uint32_t* out_false = nullptr;  // false words in input order (null: dropped)
     bool wide = false;              // 8-byte elements: n counts words (2 per element)
     uint32_t value_hi = 0;          // high word of the 8-byte value / parameter
+    // Peer publication of the kept count (sharded path): the final tile also
+    // writes board_word(count, tag) into slot (2*rank + tag%2) of every rank's
+    // count board (peer memory over NVLink / IPC); null = none.
+    uint64_t* const* pub_boards = nullptr;  // DEVICE array of `pub_world` board pointers
+    uint32_t pub_world = 0, pub_rank = 0;
+    uint64_t pub_tag = 0;
 };
+
+// Count-board word: {tag:28 | count:36}; a reader waits until the tag matches.
+constexpr int kBoardCountBits = 36;
+constexpr uint64_t kBoardTagMask = (1ull << 28) - 1;
+__host__ __device__ inline uint64_t board_word(uint64_t count, uint64_t tag) {
+    return ((tag & kBoardTagMask) << kBoardCountBits) | (count & ((1ull << kBoardCountBits) - 1));
+}
 
 struct RegArgs {
     uint32_t* ptr;
@@ -77,6 +90,10 @@ cudaError_t launch_tail_copy(uint32_t* dst_base, const uint64_t* d_offset, const
 cudaError_t launch_halo_entry(const uint32_t* ptr, size_t n, uint64_t* d_entry, cudaStream_t s);
 cudaError_t launch_shard_offsets(const uint64_t* d_counts, size_t world, size_t rank,
                                  uint64_t* d_result, cudaStream_t s);
+cudaError_t launch_publish_zero(uint64_t* const* d_boards, size_t world, size_t rank, uint64_t tag,
+                                cudaStream_t s);
+cudaError_t launch_board_offsets(const uint64_t* d_board, size_t world, size_t rank, uint64_t tag,
+                                 uint64_t* d_counts, uint64_t* d_result, cudaStream_t s);
 
 void count_launch();
 // Diagnostics buffer set by ds_debug_set_trace (null unless it covers ntiles).

@@ -66,7 +66,21 @@ struct IrregParams {
     uint64_t tlo;     // its word offset (output word j lives at tbase[tlo + j])
     uint32_t* fbase;  // same for the false words (partition), or null
     uint64_t flo;
+    uint64_t* const* pub_boards;  // peer count boards (sharded path), or null
+    uint32_t pub_world, pub_rank;
+    uint64_t pub_tag;
 };
+
+// a8 for a shard: the kept count goes straight into every rank's count board
+// (peer memory over NVLink, mapped by CUDA IPC), one release store per rank,
+// so no separate all-gather launch is needed (ds_shard_offsets_board reads it).
+__device__ __forceinline__ void publish_to_boards(const IrregParams& p, uint64_t count) {
+    const uint64_t w = board_word(count, p.pub_tag);
+    for (uint32_t r = 0; r < p.pub_world; ++r) {
+        uint64_t* slot = p.pub_boards[r] + 2 * p.pub_rank + (p.pub_tag & 1);
+        asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(slot), "l"(w) : "memory");
+    }
+}
 
 // ---- predicates (a3) ----------------------------------------------------
 // kWide: the elements are 8 bytes (two consecutive words, the low word first);
@@ -834,7 +848,10 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             if (lane == 0) {
                 trace_event(p.trace, t, 4, globaltimer());
                 meta[o].excl = excl;
-                if (t == p.ntiles - 1 && p.d_out_n) *p.d_out_n = (excl + total) >> p.wshift;  // a8
+                if (t == p.ntiles - 1) {  // a8
+                    if (p.d_out_n) *p.d_out_n = (excl + total) >> p.wshift;
+                    if (p.pub_boards) publish_to_boards(p, (excl + total) >> p.wshift);
+                }
                 mbar_arrive(&bar_resolved[o]);
             }
         }
@@ -968,6 +985,10 @@ cudaError_t launch_irregular(const IrregArgs& a, Workspace& ws, cudaStream_t s) 
     p.value_hi = a.value_hi;
     p.wshift = a.wide ? 1u : 0u;
     p.trace = debug_trace(p.ntiles);
+    p.pub_boards = a.pub_boards;
+    p.pub_world = a.pub_world;
+    p.pub_rank = a.pub_rank;
+    p.pub_tag = a.pub_tag;
     uint32_t* tptr = a.out_true ? a.out_true : a.ptr;
     const uint64_t tmis = (reinterpret_cast<uintptr_t>(tptr) >> 2) & 3u;
     p.tbase = tptr - tmis;

@@ -32,6 +32,48 @@ __global__ void shard_offsets_kernel(const uint64_t* counts, uint32_t world, uin
     }
 }
 
+// The count board's reader (the fused alternative to the NCCL all-gather of
+// the counts): wait until every rank's word for this call (slot 2r + tag%2,
+// written by that rank's DS kernel straight into this GPU's board) carries the
+// call's tag, then write all counts (d_counts, optional) and this shard's
+// offset + the global total.  Acquire at system scope pairs with the writers'
+// release; the two slots per rank let a rank publish call k+1 while a slower
+// peer still reads call k.
+__global__ void board_offsets_kernel(const uint64_t* board, uint32_t world, uint32_t rank, uint64_t tag,
+                                     uint64_t* counts, uint64_t* out) {
+    if (threadIdx.x != 0) return;
+    unsigned long long off = 0, tot = 0;
+    const uint64_t want = tag & kBoardTagMask;
+    SpinGuard guard;
+    for (uint32_t r = 0; r < world; ++r) {
+        const uint64_t* slot = board + 2 * r + (tag & 1);
+        uint64_t v;
+        uint32_t ns = 32;
+        while (true) {
+            asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(slot) : "memory");
+            if ((v >> kBoardCountBits) == want) break;
+            guard.check("count board wait");
+            __nanosleep(ns);
+            ns = ns < 1024 ? 2 * ns : 1024;
+        }
+        const uint64_t c = v & ((1ull << kBoardCountBits) - 1);
+        if (counts) counts[r] = c;
+        tot += c;
+        if (r < rank) off += c;
+    }
+    out[0] = off;
+    out[1] = tot;
+}
+
+// An empty shard launches no DS kernel, so its count (0) is published here.
+__global__ void publish_zero_kernel(uint64_t* const* boards, uint32_t world, uint32_t rank, uint64_t tag) {
+    const uint32_t r = threadIdx.x;
+    if (r < world) {
+        uint64_t* slot = boards[r] + 2 * rank + (tag & 1);
+        asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(slot), "l"(board_word(0, tag)) : "memory");
+    }
+}
+
 // Partition's second step ("move the false elements from the
 // auxiliary buffer to the tail of Array, once the true elements have been
 // shifted"): dst_base[*d_offset + j] = src[j] for j < n_total - *d_offset.
@@ -98,6 +140,20 @@ cudaError_t launch_shard_offsets(const uint64_t* d_counts, size_t world, size_t 
                                  uint64_t* d_result, cudaStream_t s) {
     count_launch();
     shard_offsets_kernel<<<1, 128, 0, s>>>(d_counts, uint32_t(world), uint32_t(rank), d_result);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_board_offsets(const uint64_t* d_board, size_t world, size_t rank, uint64_t tag,
+                                 uint64_t* d_counts, uint64_t* d_result, cudaStream_t s) {
+    count_launch();
+    board_offsets_kernel<<<1, 32, 0, s>>>(d_board, uint32_t(world), uint32_t(rank), tag, d_counts, d_result);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_publish_zero(uint64_t* const* d_boards, size_t world, size_t rank, uint64_t tag,
+                                cudaStream_t s) {
+    count_launch();
+    publish_zero_kernel<<<1, uint32_t((world + 31) / 32 * 32), 0, s>>>(d_boards, uint32_t(world), uint32_t(rank), tag);
     return cudaGetLastError();
 }
 

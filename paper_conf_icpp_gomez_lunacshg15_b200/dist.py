@@ -85,6 +85,37 @@ class LibdsLocal:
     def slide(self, shard, n, shift, stream=None):
         self.libds.ds_slide_ex(shard if n else None, n, shift, 4, stream)
 
+    # Count boards (fused count publication over peer memory).
+    def board_alloc(self, world):
+        return self.libds.ds_board_alloc(world)
+
+    def board_free(self, board):
+        self.libds.ds_board_free(board)
+
+    def board_handle(self, board):
+        return self.libds.ds_board_ipc_handle(board)
+
+    def board_open(self, handle):
+        return self.libds.ds_board_ipc_open(handle)
+
+    def board_close(self, peer):
+        self.libds.ds_board_ipc_close(peer)
+
+    def compact_pub(self, shard, remove_value, d_count, pub, stream=None):
+        self.libds.ds_compact_pub_ex(shard if shard.numel() else None, shard.numel(), remove_value, d_count,
+                                     *pub, stream)
+
+    def select_pub(self, shard, predicate, param, d_count, pub, stream=None):
+        self.libds.ds_select_pub_ex(shard if shard.numel() else None, shard.numel(), predicate, param, d_count,
+                                    *pub, stream)
+
+    def unique_pub(self, shard, d_halo, halo_len, d_count, pub, stream=None):
+        self.libds.ds_unique_pub_ex(shard if shard.numel() else None, shard.numel(), d_halo if halo_len else None,
+                                    halo_len, d_count, *pub, stream)
+
+    def board_offsets(self, board, world, rank, tag, d_counts, d_result, stream=None):
+        self.libds.ds_shard_offsets_board(board, world, rank, tag, d_counts, d_result, stream)
+
 
 class DistComm:
     """Collectives on the process group, on device tensors (NCCL on a GPU box).
@@ -172,19 +203,70 @@ class ShardResult:
 class ShardedDS:
     """One rank's view of a sharded in-place DS operation."""
 
-    def __init__(self, group=None, device=None, local=None, comm=None):
+    def __init__(self, group=None, device=None, local=None, comm=None, count_exchange="collective"):
+        """count_exchange: "collective" -- the counts travel by an all-gather
+        (NCCL); "board" -- each shard's DS kernel writes its count straight into
+        every rank's count board (peer memory mapped by CUDA IPC, NVLink between
+        GPUs) and ds_shard_offsets_board reads the local board: no all-gather
+        launch.  The board is set up once here (IPC handles exchanged over the
+        process group)."""
         self.group = group
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
         self.device = torch.device(device) if device is not None else torch.device("cuda")
         self.local = local if local is not None else LibdsLocal()
         self.comm = comm if comm is not None else DistComm(group)
+        if count_exchange not in ("collective", "board"):
+            raise ValueError("count_exchange is 'collective' or 'board'")
+        self.count_exchange = count_exchange
+        self._board = None
+        self._peers = []
+        self._tag = 0
         self.d_count = self.local.alloc_u64(1, self.device)
         self.d_counts = self.local.alloc_u64(self.world, self.device)
         self.d_result = self.local.alloc_u64(2, self.device)
         self.d_entry = self.local.alloc_u64(1, self.device)
         self.d_halo = self.local.alloc_u64(self.world, self.device)
         self._sizes = None  # every rank's shard capacity (rebalance), gathered once
+        if count_exchange == "board":
+            self._board_setup()
+
+    def _board_setup(self):
+        self._board = self.local.board_alloc(self.world)
+        handle = self.local.board_handle(self._board)
+        if self.world > 1:
+            handles = [None] * self.world
+            dist.all_gather_object(handles, handle, group=self.group)
+        else:
+            handles = [handle]
+        ptrs = []
+        for r, h in enumerate(handles):
+            if r == self.rank:
+                ptrs.append(self._board)
+            else:
+                p = self.local.board_open(h)
+                self._peers.append(p)
+                ptrs.append(p)
+        self.d_boards = torch.tensor(ptrs, dtype=torch.int64, device=self.device)
+
+    def close(self):
+        """Unmap the peers' boards and free this rank's (board mode)."""
+        if self._board is not None:
+            torch.cuda.synchronize(self.device)
+            if self.world > 1:
+                dist.barrier(group=self.group)  # no peer writes into this board any more
+            for p in self._peers:
+                self.local.board_close(p)
+            self.local.board_free(self._board)
+            self._board, self._peers = None, []
+
+    def _pub(self):
+        self._tag += 1
+        return (self.d_boards, self.world, self.rank, self._tag)
+
+    def _finish_board(self, stream) -> ShardResult:
+        self.local.board_offsets(self._board, self.world, self.rank, self._tag, self.d_counts, self.d_result, stream)
+        return ShardResult(self.d_count, self.d_result, self.d_counts)
 
     @staticmethod
     def _on(stream):
@@ -208,10 +290,16 @@ class ShardedDS:
         return ShardResult(self.d_count, self.d_result, self.d_counts)
 
     def compact(self, shard: torch.Tensor, remove_value: int, stream=None) -> ShardResult:
+        if self._board is not None:
+            self.local.compact_pub(shard, remove_value, self.d_count, self._pub(), stream)
+            return self._finish_board(stream)
         self.local.compact(shard, remove_value, self.d_count, stream)
         return self._finish(stream)
 
     def select(self, shard: torch.Tensor, predicate: int, param: int = 0, stream=None) -> ShardResult:
+        if self._board is not None:
+            self.local.select_pub(shard, predicate, param, self.d_count, self._pub(), stream)
+            return self._finish_board(stream)
         self.local.select(shard, predicate, param, self.d_count, stream)
         return self._finish(stream)
 
@@ -250,5 +338,8 @@ class ShardedDS:
         # word, but every rank must read its neighbour's value, R18).
         self.local.halo_entry(shard, self.d_entry, stream)
         self._allgather(self.d_halo, self.d_entry, stream)
+        if self._board is not None:
+            self.local.unique_pub(shard, self.d_halo, self.rank, self.d_count, self._pub(), stream)
+            return self._finish_board(stream)
         self.local.unique(shard, self.d_halo, self.rank, self.d_count, stream)
         return self._finish(stream)

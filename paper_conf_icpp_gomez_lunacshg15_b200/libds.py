@@ -22,6 +22,16 @@ DS_PRED_COUNT = 7
 _sz, _u32, _u64, _i = ctypes.c_size_t, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
 _vp = ctypes.c_void_p
 _psz = ctypes.POINTER(ctypes.c_size_t)
+_pvp = ctypes.POINTER(ctypes.c_void_p)
+
+
+class DsPublish(ctypes.Structure):
+    """ds_publish (include/ds.h): where a shard's DS kernel publishes its count."""
+    _fields_ = [("d_boards", ctypes.c_void_p), ("world", ctypes.c_size_t), ("rank", ctypes.c_size_t),
+                ("tag", ctypes.c_uint64)]
+
+
+_ppub = ctypes.POINTER(DsPublish)
 SIGNATURES = {
     "ds_pad": (_i, [_vp, _sz, _sz, _sz, _sz]),
     "ds_unpad": (_i, [_vp, _sz, _sz, _sz, _sz]),
@@ -47,6 +57,15 @@ SIGNATURES = {
     "ds_partition_copy_ex": (_i, [_vp, _sz, _i, _u32, _vp, _vp, _vp, _vp]),
     "ds_halo_entry": (_i, [_vp, _sz, _vp, _vp]),
     "ds_shard_offsets": (_i, [_vp, _sz, _sz, _vp, _vp]),
+    "ds_board_alloc": (_i, [_sz, _pvp]),
+    "ds_board_free": (_i, [_vp]),
+    "ds_board_ipc_handle": (_i, [_vp, _vp]),
+    "ds_board_ipc_open": (_i, [_vp, _pvp]),
+    "ds_board_ipc_close": (_i, [_vp]),
+    "ds_compact_pub_ex": (_i, [_vp, _sz, _u32, _vp, _ppub, _vp]),
+    "ds_select_pub_ex": (_i, [_vp, _sz, _i, _u32, _vp, _ppub, _vp]),
+    "ds_unique_pub_ex": (_i, [_vp, _sz, _vp, _sz, _vp, _ppub, _vp]),
+    "ds_shard_offsets_board": (_i, [_vp, _sz, _sz, _u64, _vp, _vp, _vp]),
     "ds_status_string": (ctypes.c_char_p, [_i]),
     "ds_last_error": (ctypes.c_char_p, []),
     "ds_release_workspaces": (_i, []),
@@ -246,6 +265,67 @@ def ds_halo_entry(ptr, n: int, d_entry, stream=None) -> None:
 def ds_shard_offsets(d_counts, world: int, rank: int, d_result, stream=None) -> None:
     _check(_lib.ds_shard_offsets(_addr(d_counts), world, rank, _addr(d_result), _stream(stream)),
            "ds_shard_offsets")
+
+
+# ------------------------------------------------------------ count boards
+DS_IPC_HANDLE_BYTES = 64
+
+
+def ds_board_alloc(world: int) -> int:
+    p = ctypes.c_void_p()
+    _check(_lib.ds_board_alloc(world, ctypes.byref(p)), "ds_board_alloc")
+    return int(p.value)
+
+
+def ds_board_free(d_board: int) -> None:
+    _check(_lib.ds_board_free(d_board), "ds_board_free")
+
+
+def ds_board_ipc_handle(d_board: int) -> bytes:
+    buf = ctypes.create_string_buffer(DS_IPC_HANDLE_BYTES)
+    _check(_lib.ds_board_ipc_handle(d_board, buf), "ds_board_ipc_handle")
+    return buf.raw
+
+
+def ds_board_ipc_open(handle: bytes) -> int:
+    if len(handle) != DS_IPC_HANDLE_BYTES:
+        raise ValueError("an IPC handle is 64 bytes")
+    p = ctypes.c_void_p()
+    _check(_lib.ds_board_ipc_open(ctypes.create_string_buffer(handle, DS_IPC_HANDLE_BYTES), ctypes.byref(p)),
+           "ds_board_ipc_open")
+    return int(p.value)
+
+
+def ds_board_ipc_close(d_peer_board: int) -> None:
+    _check(_lib.ds_board_ipc_close(d_peer_board), "ds_board_ipc_close")
+
+
+def _pub(d_boards, world, rank, tag):
+    return ctypes.byref(DsPublish(_addr(d_boards), world, rank, tag))
+
+
+def ds_compact_pub_ex(ptr, n: int, remove_value: int, d_out_n, d_boards, world: int, rank: int, tag: int,
+                      stream=None) -> None:
+    _check(_lib.ds_compact_pub_ex(_addr(ptr), n, remove_value & 0xFFFFFFFF, _addr(d_out_n),
+                                  _pub(d_boards, world, rank, tag), _stream(stream)), "ds_compact_pub_ex")
+
+
+def ds_select_pub_ex(ptr, n: int, predicate_id: int, param: int, d_out_n, d_boards, world: int, rank: int,
+                     tag: int, stream=None) -> None:
+    _check(_lib.ds_select_pub_ex(_addr(ptr), n, predicate_id, param & 0xFFFFFFFF, _addr(d_out_n),
+                                 _pub(d_boards, world, rank, tag), _stream(stream)), "ds_select_pub_ex")
+
+
+def ds_unique_pub_ex(ptr, n: int, d_halo, halo_len: int, d_out_n, d_boards, world: int, rank: int, tag: int,
+                     stream=None) -> None:
+    _check(_lib.ds_unique_pub_ex(_addr(ptr), n, _addr(d_halo), halo_len, _addr(d_out_n),
+                                 _pub(d_boards, world, rank, tag), _stream(stream)), "ds_unique_pub_ex")
+
+
+def ds_shard_offsets_board(d_board: int, world: int, rank: int, tag: int, d_counts, d_result,
+                           stream=None) -> None:
+    _check(_lib.ds_shard_offsets_board(d_board, world, rank, tag, _addr(d_counts), _addr(d_result),
+                                       _stream(stream)), "ds_shard_offsets_board")
 
 
 # ------------------------------------------------------------------ utilities

@@ -172,3 +172,20 @@ def test_wide_validation_before_device():
     assert st("ds_unique64", FAKE, 10, None) == INV                      # out_n required
     n = ctypes.c_size_t(99)
     assert st("ds_unique64", FAKE, 0, ctypes.byref(n)) == 0 and n.value == 0
+
+
+def test_count_board_validation():
+    """Count boards: argument checks need no device."""
+    assert st("ds_board_alloc", 0, None) == INV
+    assert st("ds_board_ipc_handle", None, None) == INV
+    assert st("ds_board_ipc_open", None, None) == INV
+    assert st("ds_board_ipc_close", None) == INV
+    assert st("ds_shard_offsets_board", None, 2, 0, 1, None, FAKE, None) == INV
+    assert st("ds_shard_offsets_board", FAKE, 2, 2, 1, None, FAKE, None) == INV
+    assert st("ds_compact_pub_ex", FAKE, 8, 0, None, None, None) == INV        # no ds_publish
+    pub = libds.DsPublish(0, 2, 0, 1)                                          # no board pointers
+    assert st("ds_compact_pub_ex", FAKE, 8, 0, None, ctypes.byref(pub), None) == INV
+    pub = libds.DsPublish(FAKE, 2, 2, 1)                                       # rank >= world
+    assert st("ds_select_pub_ex", FAKE, 8, 1, 0, None, ctypes.byref(pub), None) == INV
+    assert st("ds_unique_pub_ex", FAKE, 8, None, 3, None, ctypes.byref(libds.DsPublish(FAKE, 1, 0, 1)),
+              None) == INV                                                     # halo_len without a halo

@@ -113,3 +113,18 @@ def test_fake_shard_rebalance(G, fracs):
     got = full.cpu().numpy().view(np.uint32)
     assert plan.total == m
     assert np.array_equal(got[:m], host[:m])
+
+
+def test_sharded_ds_world1_board():
+    """Count-board mode without a process group (world 1: the rank's own board)."""
+    n = 1_000_003
+    a = dsgen.compact_input(n, 0.3, 4, device="cuda")
+    host = a.cpu().numpy().view(np.uint32).copy()
+    m = oracle.compact(host.copy(), 0)
+    ds = ShardedDS(device="cuda", count_exchange="board")
+    for rep in range(3):  # three calls: both slots and a reuse of the first
+        b = torch.from_numpy(host.copy().view(np.int32)).cuda() if rep else a
+        res = ds.compact(b, 0)
+        torch.cuda.synchronize()
+        assert res.result.tolist() == [0, m] and res.counts.tolist() == [m]
+    ds.close()

@@ -82,12 +82,12 @@ def _worker(rank, world, port, case, q):
         from paper_conf_icpp_gomez_lunacshg15_b200 import libds
         from paper_conf_icpp_gomez_lunacshg15_b200.dist import LibdsLocal, ShardedDS, shard_range
         torch.cuda.set_device(0)
-        kind, n, fracs, seed, use_stream = case
+        kind, n, fracs, seed, use_stream, exchange = case
         full = _global_input(kind, n, fracs, seed)
         lo, hi = shard_range(n, world, rank)
         shard = full[lo:hi].clone().cuda()
         stream = torch.cuda.Stream() if use_stream else None
-        ds = ShardedDS(device="cuda", local=LibdsLocal(), comm=StagedGlooComm())
+        ds = ShardedDS(device="cuda", local=LibdsLocal(), comm=StagedGlooComm(), count_exchange=exchange)
         if kind == "unique":
             res = ds.unique(shard, stream=stream)
         elif kind == "select":
@@ -102,6 +102,13 @@ def _worker(rank, world, port, case, q):
         counts = res.counts.tolist()
         held = ds.rebalance(shard, res, stream=stream)
         torch.cuda.synchronize()
+        if exchange == "board":  # a second call on the same board (the other slot), then unmap
+            again = shard.clone()
+            res2 = ds.compact(again, 0, stream=stream) if kind != "unique" else ds.unique(again, stream=stream)
+            torch.cuda.synchronize()
+            c2 = res2.counts.tolist()
+            assert c2[rank] == int(res2.count[0]) and res2.result.tolist() == [sum(c2[:rank]), sum(c2)]
+            ds.close()
         q.put((rank, lo, hi, cnt, result, counts, ragged, held, shard[:held].cpu().numpy().copy()))
     except Exception as e:  # pragma: no cover - reported to the parent
         q.put((rank, "error", repr(e)))
@@ -127,7 +134,7 @@ def _run(world, case):
     return sorted(out, key=lambda x: x[0])
 
 
-@pytest.mark.parametrize("world,case", [
+CASES = [
     (2, ("compact", 3_000_001, [0.5, 0.5], 41, False)),
     (3, ("compact", 2_000_003, [0.9, 0.1, 0.6], 42, True)),
     (4, ("compact", 1_000_000, [0.0, 1.0, 0.3, 0.7], 43, False)),
@@ -135,14 +142,21 @@ def _run(world, case):
     (4, ("unique", 500_001, [0.0, 0.5, 0.0, 1.0], 45, False)),
     (3, ("select", 1_500_007, [0.5, 0.5, 0.5], 46, True)),
     (4, ("compact", 5, [0.5], 47, False)),   # tiny: empty shards
-])
-def test_sharded_product_path_on_gpu(world, case):
+]
+
+
+@pytest.mark.parametrize("exchange", ["collective", "board"])
+@pytest.mark.parametrize("world,case", CASES)
+def test_sharded_product_path_on_gpu(world, case, exchange):
     """ShardedDS (LibdsLocal kernels, count / halo all-gathers, ds_shard_offsets)
     then ShardedDS.rebalance (wave-scheduled pieces + ds_slide) against the
     global oracle: ragged layout = concatenation of the shard outputs, and the
-    rebalanced layout = the single in-place DS of the whole array."""
+    rebalanced layout = the single in-place DS of the whole array.  exchange
+    "board": the counts go through the count boards (each shard's DS kernel
+    stores its count into every rank's board via CUDA IPC mappings) instead of
+    the all-gather; a second call then uses the boards' other slot."""
     kind, n, fracs, seed, _ = case
-    out = _run(world, case)
+    out = _run(world, case + (exchange,))
     full = _global_input(kind, n, fracs, seed).numpy().view(np.uint32).copy()
     if kind == "unique":
         m = oracle.unique(full)
