@@ -202,6 +202,19 @@ constexpr size_t kSmem = (size_t(kInStages) * kStageWords + kRingWords) * 4 + 12
 static_assert(kRingWords >= 0 && kRingWords % 4 == 0, "ring");
 static_assert(kThreads <= 1024, "CTA size");
 static_assert(kSlots >= kInStages, "a slot per input stage at least");
+// Partition (true + false words: a region is a whole tile, which the ring
+// rarely has room for, so its tiles stay in place) splits the same shared
+// memory into more input stages and a smaller ring.
+#ifndef DS_IRR_PART_STAGES
+#define DS_IRR_PART_STAGES 6
+#endif
+template <bool PART>
+struct SmemSplit {
+    static constexpr int kStages = PART ? DS_IRR_PART_STAGES : kInStages;
+    static constexpr int kRing = ((227 * 1024 - kStaticSmem - 128) / 4 - kStages * kStageWords) / 32 * 32;
+    static_assert(kRing >= 0 && kStages * kStageWords + kRing <= int(kSmem / 4), "shared memory split");
+    static_assert(kSlots >= kStages && kStages <= 32, "stages");
+};
 static_assert(kSlots % kResolvers == 0, "a slot is always served by the same resolver");
 static_assert(kSmem + kStaticSmem <= 227 * 1024, "shared memory");
 
@@ -487,7 +500,9 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
     // 128-byte aligned stage base (offset arithmetic keeps the shared window,
     // so the stage accesses stay LDS/STS)
     uint32_t* const smem = smem_raw + ((128u - (smem_addr(smem_raw) & 127u)) & 127u) / 4u;
-    uint32_t* const ring = smem + kInStages * kStageWords;
+    constexpr int kStagesK = SmemSplit<PART>::kStages;   // input stages of this kernel
+    constexpr int kRingK = SmemSplit<PART>::kRing;       // output-ring words of this kernel
+    uint32_t* const ring = smem + kStagesK * kStageWords;
     __shared__ __align__(8) uint64_t bar_loaded[kSlots], bar_drawn[kSlots], bar_counted[kSlots],
         bar_ranked[kSlots], bar_resolved[kSlots], bar_stored[kSlots];
     __shared__ SlotMeta meta[kSlots];
@@ -509,7 +524,7 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
         }
         s_end = 0xffffffffu;
         s_freed = 0;
-        s_stages = (1u << kInStages) - 1u;
+        s_stages = (1u << kStagesK) - 1u;
         s_alloc = 0;
         mbar_fence_init();
     }
@@ -762,11 +777,11 @@ __global__ void __launch_bounds__(kThreads, 1) irregular_kernel(const IrregParam
             const uint32_t need_t = region_true(total);
             const uint32_t need = need_t + region_false(falses);
             const uint32_t h0 = h, hp0 = hp;
-            if (hp + need > uint32_t(kRingWords)) {  // no wrapped regions: skip the ring's end
-                h += uint32_t(kRingWords) - hp;
+            if (hp + need > uint32_t(kRingK)) {  // no wrapped regions: skip the ring's end
+                h += uint32_t(kRingK) - hp;
                 hp = 0;
             }
-            const bool in_ring = h + need - meta[o].freed_snap <= uint32_t(kRingWords);
+            const bool in_ring = h + need - meta[o].freed_snap <= uint32_t(kRingK);
             const uint32_t rpos = hp;
             if (rt == 0) {
                 meta[o].ring_pos = in_ring ? rpos : kNoTile;

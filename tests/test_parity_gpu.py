@@ -673,3 +673,23 @@ def test_blocking_calls_from_threads():
         for m, m_exp, buf, exp in out:
             assert m == m_exp
             buf.assert_equals(exp, f"thread {j}")
+
+
+def test_select_copy_same_chunk_not_identity():
+    """out-of-place select with in and out in the same 16-byte
+    chunk (n <= 3, out = in + 2 words) must still write out: the identity-tile
+    skip applies only when the output IS the input (same base and phase)."""
+    for n in (1, 2):
+        for mis in (0, 1):
+            t = torch.zeros(16, dtype=torch.int32, device="cuda")
+            vals = np.array([0x11, 0x22, 0x33][:n], dtype=np.uint32)
+            t[4 + mis:4 + mis + n] = torch.from_numpy(vals.view(np.int32))
+            base = t.data_ptr()
+            src, dst = base + 4 * (4 + mis), base + 4 * (4 + mis + n)
+            d_n = torch.zeros(1, dtype=torch.int64, device="cuda")
+            libds.ds_select_copy_ex(src, n, libds.DS_PRED_NONZERO, 0, dst, d_n, None)
+            torch.cuda.synchronize()
+            got = t.cpu().numpy().view(np.uint32)
+            assert int(d_n.item()) == n
+            assert np.array_equal(got[4 + mis + n:4 + mis + 2 * n], vals), (n, mis, got)
+            assert np.array_equal(got[4 + mis:4 + mis + n], vals)   # input untouched

@@ -4,6 +4,7 @@ mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?" >> gpurun_out/smoke.log
 timeout 2400 python -m pytest tests -m gpu -q --timeout 1200 --timeout-method thread > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?" >> gpurun_out/bench.err
+timeout 600 python bench.py --steps 8 --no-rows --no-cpu --no-e2e --rebalance --count-exchange board > gpurun_out/bench_board.json 2> gpurun_out/bench_board.err
 timeout 600 python bench.py --impl reference > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
 for t in "memcheck all" "racecheck irregular" "racecheck regular" "synccheck all"; do
   set -- $t

@@ -99,6 +99,13 @@ def run(spec):
         else:
             timeit(f"unpad {R}x{NC}->{C} eb=1", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, 1, None),
                    lambda m: 2 * R * C)
+    elif op == "part":  # in-place partition through aux
+        n = 1 << 28
+        a = dsgen.select_input(n, dsgen.seed_for(5), device=dev)
+        t = dsgen.select_threshold(f) & 0xFFFFFFFF
+        aux = torch.empty_like(a)
+        timeit(f"partition 256M f={f}", a, lambda w, d: libds.ds_partition_ex(w, n, 1, t, aux, d, None),
+               lambda m: 4 * (2 * n + 2 * (n - m)))
     elif op == "pad12k":
         R, C, NC = 12000, 11999, 12000
         a = dsgen.matrix_input(R, C, NC, 4, device=dev)
