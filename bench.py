@@ -42,6 +42,12 @@ sys.path.insert(0, ROOT)
 
 METRIC = "effective GB/s (read+write) and % of HBM peak for in-place compact/pad, 1/2/4/8 B200"
 N_TOTAL = 1 << 32
+# Test mode only (tests/test_bench.py): several ranks on ONE GPU over gloo with
+# host-staged collectives and a smaller array, to exercise the N > 1 logic of
+# this script on a one-GPU box.  Never used for a reported number.
+TEST_GLOO = os.environ.get("DS_BENCH_TEST_GLOO") == "1"
+if TEST_GLOO:
+    N_TOTAL = 1 << int(os.environ.get("DS_BENCH_N_LOG2", "26"))
 FRAC = 0.5
 SEED = 0xD5201500 + 16 * 4  # dsgen.seed_for(4): C5
 WORKLOAD = "C5: sharded in-place stream compaction of 4G int32 (2^32 words), 50% kept, remove_value 0"
@@ -377,6 +383,57 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+class HostStagedComm:
+    """TEST_GLOO only: the ShardedDS collectives staged through host memory."""
+
+    def all_gather(self, out, inp):
+        import torch
+        import torch.distributed as dist
+        parts = [torch.empty_like(inp.cpu()) for _ in range(dist.get_world_size())]
+        dist.all_gather(parts, inp.cpu())
+        out.copy_(torch.cat(parts).to(out.device))
+
+    def exchange(self, sends, recvs):
+        import torch
+        import torch.distributed as dist
+        reqs, back = [], []
+        for t, peer in sends:
+            h = t.cpu()
+            back.append(None)
+            reqs.append(dist.isend(h, peer))
+            back[-1] = h
+        for t, peer in recvs:
+            h = torch.empty(t.shape, dtype=t.dtype)
+            reqs.append(dist.irecv(h, peer))
+            back.append((t, h))
+        for r in reqs:
+            r.wait()
+        for item in back:
+            if isinstance(item, tuple):
+                item[0].copy_(item[1].to(item[0].device))
+
+
+def all_gather_dev(out, inp):
+    """Device all-gather (NCCL); host-staged over gloo in TEST_GLOO mode."""
+    import torch
+    import torch.distributed as dist
+    if TEST_GLOO:
+        HostStagedComm().all_gather(out, inp)
+    else:
+        dist.all_gather_into_tensor(out, inp)
+
+
+def all_reduce_max_dev(t):
+    import torch
+    import torch.distributed as dist
+    if TEST_GLOO:
+        h = t.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.MAX)
+        t.copy_(h.to(t.device))
+    else:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+
+
 def run_libds(args):
     import torch
     import torch.distributed as dist
@@ -388,9 +445,13 @@ def run_libds(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if TEST_GLOO:
+        local = 0  # every rank on the one GPU
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if world > 1:
+    if world > 1 and TEST_GLOO:
+        dist.init_process_group("gloo")
+    elif world > 1:
         # the driver reads NCCL's communicator-init lines (nRanks) from stderr
         os.environ.setdefault("NCCL_DEBUG", "INFO")
         os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
@@ -412,7 +473,7 @@ def run_libds(args):
     flush_buf = torch.empty(1 << 27, dtype=torch.int32, device=dev)  # 512 MiB > 126 MB L2
     flush = lambda: flush_buf.sum()  # noqa: E731  (read-only flush: leaves no dirty lines)
     stream = torch.cuda.current_stream()
-    ds = ShardedDS(device=dev, count_exchange=args.count_exchange)
+    ds = ShardedDS(device=dev, count_exchange=args.count_exchange, comm=HostStagedComm() if TEST_GLOO else None)
 
     def barrier():
         if world > 1:
@@ -469,7 +530,7 @@ def run_libds(args):
     t = torch.tensor([step_ms, float(my_bytes), kern_ms, coll_ms], dtype=torch.float64, device=dev)
     if world > 1:
         allt = torch.zeros(world * 4, dtype=torch.float64, device=dev)
-        dist.all_gather_into_tensor(allt, t)
+        all_gather_dev(allt, t)
         per_rank = allt.view(world, 4).tolist()
     else:
         per_rank = [t.tolist()]
@@ -497,7 +558,7 @@ def run_libds(args):
                 rts.append(t0.elapsed_time(t1))
         mine = torch.tensor([statistics.median(rts)], dtype=torch.float64, device=dev)
         if world > 1:
-            dist.all_reduce(mine, op=dist.ReduceOp.MAX)
+            all_reduce_max_dev(mine)
         rebal = {"ms": round(float(mine.item()), 4), "held_rank0": held,
                  "note": "ShardedDS.rebalance after the compact step: wave-scheduled NCCL send/recv of "
                          "the pieces + ds_slide; host-synchronising plan; max over ranks"}
@@ -551,11 +612,11 @@ def run_libds(args):
             total_local = torch.tensor([off], dtype=torch.int64, device=dev)
             if world > 1:  # the count exchange of the sharded step (global offsets)
                 allc = torch.empty(world, dtype=torch.int64, device=dev)
-                dist.all_gather_into_tensor(allc, total_local)
+                all_gather_dev(allc, total_local)
             torch.cuda.synchronize()
             dt = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
             if world > 1:
-                dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+                all_reduce_max_dev(dt)
             if i > 0:
                 e2e_t.append(float(dt.item()))
             e2e_out = off
@@ -595,7 +656,8 @@ def run_libds(args):
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "int32", "data": "synthetic (counter-based hash, dsgen; seeded per global index)",
             "impl": "libds",
-            "config": {"workload": WORKLOAD, "n_total": N_TOTAL, "n_per_rank": n, "valid_fraction": FRAC,
+            "config": {"workload": WORKLOAD if not TEST_GLOO else "TEST MODE (gloo, one GPU): " + WORKLOAD,
+                       "n_total": N_TOTAL, "n_per_rank": n, "valid_fraction": FRAC,
                        "out_n": total_out, "parallelism": f"shard{world} (contiguous ranges)",
                        "l2": "inputs 16/N GiB per rank >> 126 MB L2; L2 also flushed by reading 512 MiB "
                              "between steps",

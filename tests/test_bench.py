@@ -55,3 +55,27 @@ def test_libds_arm_schema_plain_and_torchrun():
         assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert set(plain) == set(tr)                        # same schema under torchrun
     assert set(plain["roofline"]) == set(tr["roofline"])
+
+
+@pytest.mark.gpu
+@pytest.mark.slow
+@pytest.mark.parametrize("exchange", ["collective", "board"])
+def test_libds_arm_two_ranks_logic(exchange):
+    """The N > 1 logic of bench.py (per-rank kernel / collective times, max over
+    ranks, whole-job value, e2e, the rebalance leg) with 2 ranks on this one GPU:
+    test mode (DS_BENCH_TEST_GLOO) runs them over gloo with host-staged
+    collectives and a 2^24-word array -- NCCL itself needs one GPU per rank."""
+    env = dict(os.environ, DS_BENCH_TEST_GLOO="1", DS_BENCH_N_LOG2="24")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", "29519", os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--steps", "3", "--warmup", "3", "--no-rows", "--no-cpu", "--e2e-steps", "1",
+           "--rebalance", "--count-exchange", exchange]
+    r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
+    assert r.returncode == 0, r.stderr[-4000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]                    # rank 0 alone prints
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and len(d["per_rank"]) == 2 and d["config"]["n_total"] == 1 << 24
+    assert d["config"]["count_exchange"] == exchange and "TEST MODE" in d["config"]["workload"]
+    assert d["value"] > 0 and d["kernel_ms_max"] > 0 and d["collective_ms_max"] >= 0
+    assert d["rebalance"]["ms"] > 0 and d["e2e"]["value"] > 0
