@@ -356,6 +356,21 @@ def cpu_oracle_sample(n_sample, reps, src=None):
     return gbs, t, m
 
 
+def bench_config(world, count_exchange):
+    """The workload both arms report (identical dicts: the driver compares them)."""
+    from paper_conf_icpp_gomez_lunacshg15_b200.dist import shard_range
+    lo, hi = shard_range(N_TOTAL, world, 0)
+    return {"workload": WORKLOAD if not TEST_GLOO else "TEST MODE (gloo, one GPU): " + WORKLOAD,
+            "n_total": N_TOTAL, "n_per_rank": hi - lo, "valid_fraction": FRAC, "seed": SEED,
+            "parallelism": f"shard{world} (contiguous ranges)",
+            "l2": "inputs 16/N GiB per rank >> 126 MB L2; L2 also flushed by reading 512 MiB between steps",
+            "restore": "pristine shard restored by a D2D copy between steps, outside the events",
+            "step": ("ds_compact_pub_ex (count stored into every rank's count board over peer memory) + "
+                     "ds_shard_offsets_board" if count_exchange == "board" else
+                     "ds_compact_ex + NCCL all-gather of counts + ds_shard_offsets"),
+            "count_exchange": count_exchange}
+
+
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -375,7 +390,7 @@ def run_reference(args):
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(ms, 3), "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic (counter-based hash, dsgen)",
-            "config": {"workload": WORKLOAD, "sample_words": n_sample},
+            "config": bench_config(int(os.environ.get("WORLD_SIZE", str(args.gpus))), args.count_exchange),
             "cpu_baseline": {"value": round(value, 3), "unit": "GB/s", "cores": 1, "kind": "oracle",
                              "sample": sample},
             "e2e": {"value": round(value, 3), "unit": "GB/s", "h2d_bytes_per_step": 0,
@@ -656,16 +671,8 @@ def run_libds(args):
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "int32", "data": "synthetic (counter-based hash, dsgen; seeded per global index)",
             "impl": "libds",
-            "config": {"workload": WORKLOAD if not TEST_GLOO else "TEST MODE (gloo, one GPU): " + WORKLOAD,
-                       "n_total": N_TOTAL, "n_per_rank": n, "valid_fraction": FRAC,
-                       "out_n": total_out, "parallelism": f"shard{world} (contiguous ranges)",
-                       "l2": "inputs 16/N GiB per rank >> 126 MB L2; L2 also flushed by reading 512 MiB "
-                             "between steps",
-                       "restore": "pristine shard restored by a D2D copy between steps, outside the events",
-                       "step": ("ds_compact_pub_ex (count stored into every rank's count board over peer "
-                                "memory) + ds_shard_offsets_board" if args.count_exchange == "board" else
-                                "ds_compact_ex + NCCL all-gather of counts + ds_shard_offsets"),
-                       "count_exchange": args.count_exchange},
+            "config": bench_config(world, args.count_exchange),
+            "out_n": total_out,
             "frac_of_peak": round(value / world / peak, 4),
             "frac_of_nominal": round(value / world / NOMINAL_HBM_GBS, 4),
             "elems_per_s": round(N_TOTAL / (ms_per_step * 1e-3), 1),

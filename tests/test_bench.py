@@ -29,6 +29,9 @@ def test_reference_arm_on_cpu():
     assert d["impl"] == "reference" and d["unit"] == "GB/s" and d["value"] > 0
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] == 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0
+    sys.path.insert(0, ROOT)
+    import bench
+    assert d["config"] == bench.bench_config(1, "collective")   # the same config dict as the libds arm
 
 
 def _libds_line(cmd):
@@ -55,6 +58,10 @@ def test_libds_arm_schema_plain_and_torchrun():
         assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert set(plain) == set(tr)                        # same schema under torchrun
     assert set(plain["roofline"]) == set(tr["roofline"])
+    assert plain["config"] == tr["config"]
+    sys.path.insert(0, ROOT)
+    import bench
+    assert plain["config"] == bench.bench_config(1, "collective")   # what the reference arm reports
 
 
 @pytest.mark.gpu

@@ -21,7 +21,7 @@ def main():
     eb = int(sys.argv[5]) if len(sys.argv) > 5 else 4
     global T
     if eb in (1, 2) and (C * eb) % 4:  # byte-granular kernel: 32 KB output tiles
-        T = 32768 // eb
+        T = (32768 if R * max(C, NC) * eb >= (64 << 20) else 16384) // eb
     if eb == 4:
         src = dsgen.matrix_input(R, C, NC, 4, device="cuda")
     else:
