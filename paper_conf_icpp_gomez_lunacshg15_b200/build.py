@@ -36,6 +36,12 @@ VARIANTS = {
     "spincap": ("libds_spincap.so", ["-DDS_SPIN_CAP_NS=2000000000ull"]),
     # the same with tile 5 of every irregular launch never publishing (test only)
     "hang": ("libds_hang.so", ["-DDS_SPIN_CAP_NS=200000000ull", "-DDS_DEBUG_DROP_TILE=5u"]),
+    # irregular shared-memory layouts at the edges (tests): no output ring (every
+    # tile compacted in place), a ring of about one tile (wrap-around skips and a
+    # mix of ring / in place), and two input stages
+    "ring0": ("libds_ring0.so", ["-DDS_IRR_RING_WORDS=0"]),
+    "ring8k": ("libds_ring8k.so", ["-DDS_IRR_RING_WORDS=8704"]),
+    "stages2": ("libds_stages2.so", ["-DDS_IRR_IN_STAGES=2", "-DDS_IRR_PART_STAGES=2"]),
 }
 
 

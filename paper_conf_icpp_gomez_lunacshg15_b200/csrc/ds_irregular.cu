@@ -210,8 +210,11 @@ static_assert(kSlots >= kInStages, "a slot per input stage at least");
 #endif
 template <bool PART>
 struct SmemSplit {
-    static constexpr int kStages = PART ? DS_IRR_PART_STAGES : kInStages;
-    static constexpr int kRing = ((227 * 1024 - kStaticSmem - 128) / 4 - kStages * kStageWords) / 32 * 32;
+    static constexpr int kFit = int((kSmem - 128) / 4) / kStageWords;  // stages the memory holds
+    static constexpr int kStages = PART ? (DS_IRR_PART_STAGES < kFit ? DS_IRR_PART_STAGES : kFit) : kInStages;
+    // the rest of the kernel's dynamic shared memory (the same size for both)
+    static constexpr int kRingRaw = (int((kSmem - 128) / 4) - kStages * kStageWords) / 32 * 32;
+    static constexpr int kRing = PART ? (kRingRaw > 0 ? kRingRaw : 0) : kRingWords;
     static_assert(kRing >= 0 && kStages * kStageWords + kRing <= int(kSmem / 4), "shared memory split");
     static_assert(kSlots >= kStages && kStages <= 32, "stages");
 };
