@@ -197,6 +197,25 @@ def bench_rows(peak, flush):
         del bufs
         return summarize([t / copies for t in ts])
 
+    def graph_time(call, base, reps=20):
+        """One call captured in a CUDA graph on a side stream (workspace made by a
+        warm-up call there first), replayed on a restored, L2-flushed input:
+        the device time without the host's launch path."""
+        gs = torch.cuda.Stream()
+        work = torch.empty_like(base)
+        gs.wait_stream(s)
+        with torch.cuda.stream(gs):
+            work.copy_(base)
+            call(work)
+        s.wait_stream(gs)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=gs):
+            call(work)
+        ts = timed(lambda: g.replay(), s, restore=lambda: work.copy_(base), flush=flush, reps=reps)
+        del g, work
+        return summarize(ts)
+
     def regular(op, name, src, call, nbytes, reps=5, restore_src=None, batch=False):
         work = torch.empty_like(src)
         base = restore_src if restore_src is not None else src
@@ -204,8 +223,11 @@ def bench_rows(peak, flush):
         extra = None
         if batch:
             b = batched(call, base)
+            gr = graph_time(call, base)
             extra = {"back_to_back": {**b, "gbs": round(nbytes / (b["us"] * 1e-6) / 1e9, 1),
-                                      "frac": round(nbytes / (b["us"] * 1e-6) / 1e9 / peak, 4)}}
+                                      "frac": round(nbytes / (b["us"] * 1e-6) / 1e9 / peak, 4)},
+                     "graph_replay": {**gr, "gbs": round(nbytes / (gr["us"] * 1e-6) / 1e9, 1),
+                                      "frac": round(nbytes / (gr["us"] * 1e-6) / 1e9 / peak, 4)}}
         row(op, name, ts, nbytes, extra)
 
     # C1: 1M int32 compaction, 50 %: kernel time flushed and L2-hot, the blocking
@@ -234,13 +256,16 @@ def bench_rows(peak, flush):
         oracle.compact(hcopy, 0)
         ot.append(time.perf_counter() - t0)
     b2b = batched(lambda w: libds.ds_compact_ex(w, n, 0, d_n, None), src, copies=20)
+    gr = graph_time(lambda w: libds.ds_compact_ex(w, n, 0, d_n, torch.cuda.current_stream()), src)
     row("compact", "C1 1M int32 f=0.5", ts, 4 * (n + m),
         {"n": n, "out_n": m, "l2_hot": summarize(ts_hot), "blocking_wall": summarize(wall),
          "back_to_back": {**b2b, "gbs": round(4 * (n + m) / (b2b["us"] * 1e-6) / 1e9, 1)},
+         "graph_replay": {**gr, "gbs": round(4 * (n + m) / (gr["us"] * 1e-6) / 1e9, 1)},
          "oracle_s": round(statistics.median(ot), 6),
          "note": "flushed: 512 MiB read between reps; l2_hot: input restored by a D2D copy only "
                  "(it stays in L2); blocking_wall: ds_compact (legacy stream) incl. the D2H of out_n; "
-                 "back_to_back: 20 calls on 20 restored copies between the events, per call"})
+                 "back_to_back: 20 calls on 20 restored copies between the events, per call; graph_replay: "
+                 "the call captured in a CUDA graph, one replay between the events"})
     del src, work
     # C2: pad 4000x3990 -> 4000 f32 and unpad back
     R, C, NC = 4000, 3990, 4000

@@ -56,6 +56,11 @@
  *    the data) and one ticket/epoch word.  Calls that share a stream share it; calls on
  *    different streams may run concurrently.  ds_release_workspaces()
  *    frees it (call only when no libds kernel is in flight).
+ *  - CUDA graphs: once a stream's workspace exists (after one call on it),
+ *    the _ex forms on that stream may be captured: they do not synchronise
+ *    or allocate, and every launch re-arms its own ticket word (R24).  The
+ *    host zeroes the status words every 2^25 launches it issues; a graph
+ *    replayed more than 2^25 times should be re-captured.
  *  - Thread-safe: host state (workspaces, launch parameters) is protected
  *    by a mutex held only while a call validates and enqueues its kernels.
  *    Every blocking call reads its count through a count word of its own
