@@ -740,7 +740,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=2)
-    ap.add_argument("--e2e-chunks", type=int, default=32)
+    ap.add_argument("--e2e-chunks", type=int, default=256)
     ap.add_argument("--rebalance", action="store_true", help="also time ShardedDS.rebalance (8(f)-1)")
     ap.add_argument("--count-exchange", default="collective", choices=["collective", "board"],
                     help="counts by NCCL all-gather (default) or through the count boards (peer memory)")
