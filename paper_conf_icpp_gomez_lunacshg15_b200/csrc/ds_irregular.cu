@@ -189,6 +189,14 @@ struct Layout {
     static constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;
     static constexpr int kThreads = 32 * (kWarpProducer + 1);
     static_assert(kThreads <= 1024, "CTA size");
+#ifndef DS_IRR_REPHASE_CHUNKS
+#define DS_IRR_REPHASE_CHUNKS 384
+#endif
+#ifndef DS_IRR_PART_REPHASE_CHUNKS
+#define DS_IRR_PART_REPHASE_CHUNKS 384
+#endif
+    static constexpr int kRephaseChunks = PART ? DS_IRR_PART_REPHASE_CHUNKS : DS_IRR_REPHASE_CHUNKS;
+    static constexpr int kRephaseU = kRephaseChunks / kST > 0 ? kRephaseChunks / kST : 1;
 };
 // Words before the tile in a stage (unique's boundary words).  Stages, and the
 // tile inside each stage, start on 128-byte boundaries, so a bulk copy fills
@@ -421,9 +429,11 @@ __device__ __forceinline__ void store_segment(uint32_t* base, uint64_t d0, uint3
 // [4c, 4c+4)) takes source words [4c-ph, 4c+4-ph): two aligned vector loads.
 // Writing chunk c destroys sources of chunk c+1 only, so the chunks go in
 // descending rounds, each reading everything before writing.
-template <int kSTT>
+// kU chunks per thread per round: 384 chunks per round is the measured
+// optimum for both 96 storers (kU = 4; compaction 1G f = 0.5: kU = 2 / 4 / 8
+// 79.3 / 83.8 / 77.6 %) and 192 (partition, kU = 2: 75.7 %, kU = 4 73.6 %).
+template <int kSTT, int kU>
 __device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph, int st) {
-    constexpr int kU = 4;
     const int32_t nchunks = int32_t((cnt + ph + 3) >> 2);
     for (int32_t hi = nchunks; hi > 0; hi -= kU * kSTT) {
         const int32_t lo = hi - kU * kSTT;
@@ -919,7 +929,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             auto bulk_segment = [&](uint32_t* w0, uint32_t* base, uint64_t d0, uint32_t cnt) {
                 const uint64_t d1 = d0 + cnt;
                 const uint32_t sh = uint32_t(d0) & 3u;  // word r must sit at phase (d0 + r) & 3
-                if (sh) rephase<kST>(w0, cnt, sh, st);
+                if (sh) rephase<kST, Layout<PART>::kRephaseU>(w0, cnt, sh, st);
                 const uint32_t* const w = w0 + sh;
                 const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
                 if (g1 > g0) {
