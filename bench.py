@@ -389,7 +389,8 @@ def bench_config(world, count_exchange):
             "n_total": N_TOTAL, "n_per_rank": hi - lo, "valid_fraction": FRAC, "seed": SEED,
             "parallelism": f"shard{world} (contiguous ranges)",
             "l2": "inputs 16/N GiB per rank >> 126 MB L2; L2 also flushed by reading 512 MiB between steps",
-            "restore": "pristine shard restored by a D2D copy between steps, outside the events",
+            "restore": "pristine shard restored by a D2D copy between steps, outside the events "
+                       "(the prefix [0, out_n) the compaction rewrites; the tail is checked untouched once)",
             "step": ("ds_compact_pub_ex (count stored into every rank's count board over peer memory) + "
                      "ds_shard_offsets_board" if count_exchange == "board" else
                      "ds_compact_ex + NCCL all-gather of counts + ds_shard_offsets"),
@@ -534,14 +535,24 @@ def run_libds(args):
             ds._finish(stream)
         c.record(stream)
 
+    # The compaction writes only words [0, out_n) (R5: the tail keeps its
+    # bytes), so once out_n is known the restore copies that prefix alone; the
+    # first warm-up step restores everything and checks the tail is untouched.
+    restore_n = [n]
+
     def one_step(timed_events):
-        work.copy_(pristine)
+        work[:restore_n[0]].copy_(pristine[:restore_n[0]])
         flush()
         step_once(timed_events)
 
     # ---- warm-up
-    for _ in range(args.warmup):
+    for i in range(args.warmup):
         one_step([torch.cuda.Event(enable_timing=True) for _ in range(3)])
+        if i == 0:
+            m = int(ds.d_count.item())
+            if not torch.equal(work[m:], pristine[m:]):
+                raise SystemExit("bench: compaction changed words past out_n")
+            restore_n[0] = m
     barrier()
 
     # ---- timed region: exactly K steps, barrier + sync on both sides

@@ -32,7 +32,10 @@ constexpr int kBCT = 32 * kBConsumerWarps;
 // matrices; 16 KB tiles when the output is small (< kSmallOut), where 32 KB
 // tiles leave too few tiles per CTA to fill the pipeline (1-byte pad at the C2
 // shape 19.5 -> 15.4 us; at 16384 x 16384 16 KB tiles cost 15 %).
-constexpr int kTBLarge = 32768, kTBSmall = 16384;
+#ifndef DS_REGB_SMALL_TILE
+#define DS_REGB_SMALL_TILE 16384
+#endif
+constexpr int kTBLarge = 32768, kTBSmall = DS_REGB_SMALL_TILE;
 constexpr uint64_t kSmallOut = 64ull << 20;
 template <int TB>
 struct BCfg {
