@@ -55,7 +55,11 @@
  *    status word per tile of 8192 words (one per 64-byte line, ~0.2% of
  *    the data) and one ticket/epoch word.  Calls that share a stream share it; calls on
  *    different streams may run concurrently.  ds_release_workspaces()
- *    frees it (call only when no libds kernel is in flight).
+ *    frees it (call only when no libds kernel is in flight).  The key is
+ *    the stream handle, and CUDA may hand a destroyed stream's handle to a
+ *    new stream: synchronise a stream that ran libds calls before
+ *    destroying it, or a new stream could share its workspace while those
+ *    calls are still running.
  *  - CUDA graphs: once a stream's workspace exists (after one call on it),
  *    the _ex forms on that stream may be captured: they do not synchronise
  *    or allocate, and every launch re-arms its own ticket word (R24).  The
@@ -205,9 +209,11 @@ ds_status ds_unique64_ex(void* ptr, size_t n, uint64_t* d_out_n, ds_stream_t str
  * then the false words, both in input order.  As in the paper, the false
  * words go through an auxiliary buffer ("Array_false should be an
  * auxiliary buffer"): `aux` is a caller-owned DEVICE buffer of at
- * least n words; libds allocates nothing n-sized.  One DS pass slides the
+ * least n words, not overlapping ptr[0, n) (DS_ERROR_INVALID_VALUE
+ * otherwise); libds allocates nothing n-sized.  One DS pass slides the
  * trues in place and writes the falses to aux in order, then a copy moves
- * them to the tail ptr[*out_n_true, n).  out_n_true: HOST, required.      */
+ * them to the tail ptr[*out_n_true, n); aux[0, n - *out_n_true) is
+ * overwritten.  out_n_true: HOST, required.                              */
 ds_status ds_partition(void* ptr, size_t n, int predicate_id, void* aux, size_t* out_n_true);
 /* Asynchronous form; d_out_n_true (DEVICE, required) receives the true count. */
 ds_status ds_partition_ex(void* ptr, size_t n, int predicate_id, uint32_t param, void* aux,
@@ -216,13 +222,14 @@ ds_status ds_partition_ex(void* ptr, size_t n, int predicate_id, uint32_t param,
 /* ds_select_copy_ex -- out-of-place select ("DS Copy_if"):
  * the predicate-true words of in[0, n) are written in order to out[0, count);
  * in is not modified.  out == in gives the in-place select; otherwise the
- * two buffers must not overlap.                                          */
+ * two n-word ranges must not overlap (DS_ERROR_INVALID_VALUE).           */
 ds_status ds_select_copy_ex(const void* in, size_t n, int predicate_id, uint32_t param,
                             void* out, uint64_t* d_out_n, ds_stream_t stream);
 
 /* ds_partition_copy_ex -- out-of-place stable partition: trues to
  * out_true[0, t), falses to out_false[0, n - t); in is not modified; the
- * three buffers must not overlap.  d_out_n_true: DEVICE, may be NULL.    */
+ * three n-word ranges must not overlap (DS_ERROR_INVALID_VALUE).
+ * d_out_n_true: DEVICE, may be NULL.                                     */
 ds_status ds_partition_copy_ex(const void* in, size_t n, int predicate_id, uint32_t param,
                                void* out_true, void* out_false, uint64_t* d_out_n_true,
                                ds_stream_t stream);

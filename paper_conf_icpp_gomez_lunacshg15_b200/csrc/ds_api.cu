@@ -48,6 +48,12 @@ ds_status fail(cudaError_t e, const char* what) {
 
 bool misaligned(const void* p, uintptr_t a) { return (reinterpret_cast<uintptr_t>(p) & (a - 1)) != 0; }
 
+// Do the n-word ranges at a and b share a byte?  (n <= kMaxWords, so no overflow.)
+bool overlap(const void* a, const void* b, size_t n) {
+    const uintptr_t x = reinterpret_cast<uintptr_t>(a), y = reinterpret_cast<uintptr_t>(b);
+    return n > 0 && x < y + 4 * n && y < x + 4 * n;
+}
+
 // Caller holds g_mu.
 ds_status get_workspace(size_t tiles, cudaStream_t s, ds::Workspace** out) {
     int dev = 0;
@@ -463,6 +469,7 @@ ds_status ds_select_copy_ex(const void* in, size_t n, int predicate_id, uint32_t
     ds_status st = check_irregular(in, n, d_out_n);
     if (st != DS_SUCCESS) return st;
     if (n > 0 && (!out || misaligned(out, 4))) return DS_ERROR_INVALID_VALUE;
+    if (out != in && overlap(in, out, n)) return DS_ERROR_INVALID_VALUE;  // in place only at out == in
     ds::IrregArgs a{const_cast<uint32_t*>(static_cast<const uint32_t*>(in)), n, ds::IrregOp::Select,
                     predicate_id, param, nullptr, 0, d_out_n};
     a.out_true = static_cast<uint32_t*>(out);
@@ -476,6 +483,8 @@ ds_status ds_partition_copy_ex(const void* in, size_t n, int predicate_id, uint3
     ds_status st = check_irregular(in, n, d_out_n_true);
     if (st != DS_SUCCESS) return st;
     if (n > 0 && (!out_true || !out_false || misaligned(out_true, 4) || misaligned(out_false, 4)))
+        return DS_ERROR_INVALID_VALUE;
+    if (overlap(in, out_true, n) || overlap(in, out_false, n) || overlap(out_true, out_false, n))
         return DS_ERROR_INVALID_VALUE;
     ds::IrregArgs a{const_cast<uint32_t*>(static_cast<const uint32_t*>(in)), n, ds::IrregOp::Select,
                     predicate_id, param, nullptr, 0, d_out_n_true};
@@ -491,6 +500,7 @@ ds_status ds_partition_ex(void* ptr, size_t n, int predicate_id, uint32_t param,
     ds_status st = check_irregular(ptr, n, d_out_n_true);
     if (st != DS_SUCCESS) return st;
     if (n > 0 && (!aux || misaligned(aux, 4))) return DS_ERROR_INVALID_VALUE;
+    if (overlap(ptr, aux, n)) return DS_ERROR_INVALID_VALUE;
     if (n == 0) return irregular_ex(ds::IrregArgs{static_cast<uint32_t*>(ptr), 0, ds::IrregOp::Select,
                                                   predicate_id, param, nullptr, 0, d_out_n_true},
                                     reinterpret_cast<cudaStream_t>(stream));
@@ -513,6 +523,7 @@ ds_status ds_partition(void* ptr, size_t n, int predicate_id, void* aux, size_t*
     ds_status st = check_irregular(ptr, n, nullptr);
     if (st != DS_SUCCESS) return st;
     if (n > 0 && (!aux || misaligned(aux, 4))) return DS_ERROR_INVALID_VALUE;
+    if (overlap(ptr, aux, n)) return DS_ERROR_INVALID_VALUE;
     if (n == 0) {
         *out_n_true = 0;
         return DS_SUCCESS;

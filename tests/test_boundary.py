@@ -149,6 +149,13 @@ def test_partition_and_copy_validation():
     assert st("ds_select_copy_ex", FAKE, 10, 0, 0, None, None, None) == INV  # no out
     assert st("ds_select_copy_ex", FAKE, 10, 0, 0, BAD, None, None) == INV   # misaligned out
     assert st("ds_partition_copy_ex", FAKE, 10, 0, 0, FAKE, None, None, None) == INV
+    # overlapping buffers are rejected before the device is touched
+    W = FAKE + 0x10000
+    assert st("ds_partition", FAKE, 10, 0, FAKE + 36, out_sz()) == INV            # aux inside ptr[0, 10)
+    assert st("ds_partition_ex", FAKE, 10, 0, 0, FAKE - 36, W, None) == INV        # aux ends inside ptr
+    assert st("ds_select_copy_ex", FAKE, 10, 0, 0, FAKE + 4, None, None) == INV    # shifted by one word
+    assert st("ds_partition_copy_ex", FAKE, 10, 0, 0, W, W + 8, None, None) == INV  # true / false overlap
+    assert st("ds_partition_copy_ex", FAKE, 10, 0, 0, FAKE, W, None, None) == INV   # out_true == in
 
 
 def test_slide_validation_before_device():
