@@ -298,9 +298,10 @@ uint64_t ds_launch_count(void);
  * `capacity_tiles` records 16 uint64 per tile into the DEVICE buffer d_trace
  * (globaltimer ns: 0 drawn, 1 landed, 2 aggregate published, 3 look-back
  * start, 4 prefix published, 5 stores start, 6 stores issued; 7 SM id;
- * 8 look-back rounds, 9 polls, 10 first round read, 11 resolved, 12 after
- * the acquire fence; 13 the producer starts waiting for a free input stage,
- * 14 after the ranker barrier; 7 also carries bit 16 = compacted into the
+ * 8 look-back rounds, 9 polls, 10 first round read, 11 resolved, 12 the
+ * bulk engine has read the stored region (irregular; region released);
+ * 13 the producer starts waiting for a free input stage, 14 after the
+ * ranker barrier, 15 compacted; 7 also carries bit 16 = compacted into the
  * output ring (else in place)).
  * NULL disables.  Development aid for DESIGN.md §7, not used by the API.  */
 ds_status ds_debug_set_trace(uint64_t* d_trace, size_t capacity_tiles);

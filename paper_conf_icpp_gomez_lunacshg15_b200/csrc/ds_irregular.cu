@@ -369,7 +369,6 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
     }
     lookback_acquire();
     __syncwarp();
-    if (lane == 0) trace_event(trace, tile, 12, globaltimer());
     return excl;
 }
 
@@ -961,6 +960,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
                 trace_event(p.trace, t, 6, globaltimer());
                 bulk_commit();        // (possibly empty) group of this tile
                 bulk_wait_read<0>();  // the bulk engine has read the region
+                trace_event(p.trace, t, 12, globaltimer());
                 // ring words allocated up to this tile belong to tiles stored by now
                 st_release_cta_smem(&s_freed, ring_end);
                 if (!in_ring) stage_release(&s_stages, meta[o].stage);

@@ -58,7 +58,7 @@ def main():
         print(f"{name:9s} p5 {q[0]:7.2f}  p50 {q[1]:7.2f}  p95 {q[2]:7.2f}  p99 {q[3]:7.2f}  mean {d.mean():7.2f}")
     lb = (t[:, [10, 11, 12]] - t0) / 1e3
     for name, d in (("lb:first-read", lb[:, 0] - ev[:, 3]), ("lb:resolve", lb[:, 1] - lb[:, 0]),
-                    ("lb:fence", lb[:, 2] - lb[:, 1]), ("lb:publish", ev[:, 4] - lb[:, 2])):
+                    ("lb:publish", ev[:, 4] - lb[:, 1])):
         q = np.percentile(d[1:], [5, 50, 95, 99])
         print(f"{name:13s} p5 {q[0]:7.2f}  p50 {q[1]:7.2f}  p95 {q[2]:7.2f}  p99 {q[3]:7.2f}")
     sub = (t[:, [1, 13, 14, 2]] - t0) / 1e3
