@@ -3,8 +3,8 @@
 // §III-B; primitives §IV-B/C P:230-282).
 //
 // One persistent, warp-specialised CTA per SM walks input tiles of
-// T = 8192 words in dynamic-ticket order (Fig. 4) through 4 input stages and
-// an output ring in shared memory.  Each role works on a different tile:
+// T = 8192 words in dynamic-ticket order (Fig. 4) through 4 input stages
+// (partition: 6) and an output ring in shared memory.  Each role works on a different tile:
 //
 //   producer warp    a1 draws the next ticket as soon as an input stage and a
 //                       slot are free; a2 loads the tile (plus, for unique,
@@ -18,15 +18,16 @@
 //                       input order ("binary prefix sum": one
 //                       shuffle scan over packed per-lane counts) and the
 //                       compaction of the kept words into the output ring
-//   8 resolver warps a5 decoupled look-back over 32 predecessors per round
-//                       trip, started as soon as the ticket is drawn (it needs
-//                       no data), then INCL; the last tile writes out_n (a8).
-//                       This replaces the serial flag chain of Fig. 7, which is
-//                       latency-bound on B200
-//   5 storer warps   a7 re-phase the tile's ring region to the destination's
-//                       16-byte phase, one TMA bulk store of [excl, excl + A)
+//   3 resolver warps a5 decoupled look-back over 32 predecessors per round
+//                       trip, started once the tile's own AGG is out, then
+//                       INCL; the last tile writes out_n (a8).  This replaces
+//                       the serial flag chain of Fig. 7, which is latency-bound
+//                       on B200
+//   2 x 2 storer     a7 re-phase the tile's ring region to the destination's
+//     warps             16-byte phase, one TMA bulk store of [excl, excl + A)
 //                       (scalar head/tail), then free the region once the bulk
-//                       engine has read it
+//                       engine has read it; two groups on alternate tiles,
+//                       regions released in ring order (partition: 2 x 3)
 //
 // A drawn tile's AGG depends only on its own load and ranking, never on the
 // resolution of earlier tiles.  In-place safety: AGG/INCL
@@ -130,18 +131,18 @@ struct OpUnique64 {
 };
 
 // ---- CTA shape ----------------------------------------------------------
-// warps: 16 rankers (2 groups of 8) | 4 resolvers | 3 storers (6 for partition) | 1 producer
+// warps: 16 rankers (2 groups of 8) | 3 resolvers | 2 x 2 storers (2 x 3 for partition) | 1 producer
 #ifndef DS_IRR_IN_STAGES
 #define DS_IRR_IN_STAGES 4
 #endif
 #ifndef DS_IRR_SLOTS
-#define DS_IRR_SLOTS 16
+#define DS_IRR_SLOTS 18
 #endif
 #ifndef DS_IRR_RESOLVERS
-#define DS_IRR_RESOLVERS 4
+#define DS_IRR_RESOLVERS 3
 #endif
 #ifndef DS_IRR_STORE_WARPS
-#define DS_IRR_STORE_WARPS 3
+#define DS_IRR_STORE_WARPS 2
 #endif
 #ifndef DS_IRR_BULK_STORE
 #define DS_IRR_BULK_STORE 1
@@ -175,15 +176,27 @@ constexpr int kInStages = DS_IRR_IN_STAGES;   // input tiles (TMA destination)
 constexpr int kSlots = DS_IRR_SLOTS;          // tiles in flight per CTA (meta ring)
 constexpr int kResolvers = DS_IRR_RESOLVERS;  // resolver r serves ring positions k = r mod kResolvers
 #ifndef DS_IRR_PART_STORE_WARPS
-#define DS_IRR_PART_STORE_WARPS 6
+#define DS_IRR_PART_STORE_WARPS 3
 #endif
-// Warp layout: rankers | resolvers | storers | producer.  Partition stores two
-// segments per tile (trues and falses) and gets more storer warps (6 instead of
-// 3: partition 256M f = 0.1 / 0.5 68.5 -> 73.4 % / 71.4 -> 73.6 %).
+#ifndef DS_IRR_STORE_GROUPS
+#define DS_IRR_STORE_GROUPS 2
+#endif
+#ifndef DS_IRR_PART_STORE_GROUPS
+#define DS_IRR_PART_STORE_GROUPS 2
+#endif
+// Warp layout: rankers | resolvers | storers | producer.  The storers form
+// kStoreGroups groups of kGroupStoreWarps warps; group g stores the tiles at
+// ring positions k = g (mod kStoreGroups), so one group's per-tile fixed costs
+// (re-phase, barriers, bulk issue, head / tail words) overlap the other's, and
+// the regions are released in ring order (s_released).  Partition stores two
+// segments per tile (trues and falses) and gets more storer warps.
 template <bool PART>
 struct Layout {
-    static constexpr int kStoreWarps = PART ? DS_IRR_PART_STORE_WARPS : DS_IRR_STORE_WARPS;
-    static constexpr int kST = 32 * kStoreWarps;
+    static constexpr int kStoreGroups = PART ? DS_IRR_PART_STORE_GROUPS : DS_IRR_STORE_GROUPS;
+    static constexpr int kGroupStoreWarps = PART ? DS_IRR_PART_STORE_WARPS : DS_IRR_STORE_WARPS;
+    static constexpr int kStoreWarps = kStoreGroups * kGroupStoreWarps;
+    static constexpr int kST = 32 * kGroupStoreWarps;  // threads of one storer group
+    static_assert(kStoreGroups == 1 || kStoreGroups == 2, "named barriers 2 and 4 serve the storer groups");
     static constexpr int kWarpResolver0 = kRankWarps;
     static constexpr int kWarpStorer0 = kRankWarps + kResolvers;
     static constexpr int kWarpProducer = kWarpStorer0 + kStoreWarps;
@@ -208,7 +221,7 @@ constexpr int kStageWords = kT + kPre + 32;
 // ring (the stage is free as soon as every ranker holds its words in
 // registers); the storers drain the ring in tile order once the prefix is
 // known.  Everything left of the 227 KB after the input stages.
-constexpr int kStaticSmem = 128 * kSlots + 512;  // barriers + slot metadata (static shared memory; ptxas: 2048 B at 16 slots)
+constexpr int kStaticSmem = 128 * kSlots + 512;  // barriers + slot metadata (static shared memory; ptxas: 2304 B at 18 slots)
 #ifndef DS_IRR_RING_WORDS
 #define DS_IRR_RING_WORDS (((227 * 1024 - kStaticSmem - 128) / 4 - kInStages * kStageWords) / 32 * 32)
 #endif
@@ -432,7 +445,7 @@ __device__ __forceinline__ void store_segment(uint32_t* base, uint64_t d0, uint3
 // optimum for both 96 storers (kU = 4; compaction 1G f = 0.5: kU = 2 / 4 / 8
 // 79.3 / 83.8 / 77.6 %) and 192 (partition, kU = 2: 75.7 %, kU = 4 73.6 %).
 template <int kSTT, int kU>
-__device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph, int st) {
+__device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph, int st, uint32_t bar) {
     const int32_t nchunks = int32_t((cnt + ph + 3) >> 2);
     for (int32_t hi = nchunks; hi > 0; hi -= kU * kSTT) {
         const int32_t lo = hi - kU * kSTT;
@@ -453,13 +466,66 @@ __device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph
                 }
             }
         }
-        named_bar_sync(2, kSTT);
+        named_bar_sync(bar, kSTT);
 #pragma unroll
         for (int u = 0; u < kU; ++u) {
             const int32_t c = lo + u * kSTT + st;
             if (c >= 0 && c < hi) *reinterpret_cast<u32x4*>(seg + 4 * c) = w[u];
         }
-        named_bar_sync(2, kSTT);
+        named_bar_sync(bar, kSTT);
+    }
+}
+
+// a7 helper, one-barrier form of rephase(): every thread takes a contiguous
+// run of m destination chunks (m odd, so the 16-byte accesses of 8
+// neighbouring threads fall in distinct bank groups) and walks it downwards.
+// Destination chunk c needs source chunks c-1 and c; writing it destroys
+// source c only, which no lower chunk needs.  Within a run the walk order
+// keeps every source intact until read; the one source a run needs from
+// below its own range (chunk c_lo - 1, the next-lower run's top) is read
+// before the barrier.  No barrier at the end: the caller's fence + barrier
+// before the bulk store orders the writes.
+#ifndef DS_IRR_STORE_WARP_SYNC
+#define DS_IRR_STORE_WARP_SYNC 1
+#endif
+#ifndef DS_IRR_REPHASE_RUNS
+#define DS_IRR_REPHASE_RUNS 1
+#endif
+template <int kSTT>
+__device__ __forceinline__ void rephase_runs(uint32_t* seg, uint32_t cnt, uint32_t ph, int st,
+                                             uint32_t bar) {
+    const int32_t nchunks = int32_t((cnt + ph + 3) >> 2);
+    const int32_t m = ((nchunks + kSTT - 1) / kSTT) | 1;
+    const int32_t c_lo = st * m;
+    const int32_t c_hi = c_lo + m < nchunks ? c_lo + m : nchunks;
+    // chunk 0's leading words are dead (never stored): its "lower" source is
+    // chunk 0 itself, since the words before seg may belong to another region
+    u32x4 below = u32x4{0u, 0u, 0u, 0u};
+    if (c_lo < nchunks) below = *reinterpret_cast<const u32x4*>(seg + 4 * (c_lo > 0 ? c_lo - 1 : 0));
+    named_bar_sync(bar, kSTT);
+    if (c_lo >= c_hi) return;
+    auto comb = [ph](const u32x4& a, const u32x4& b) {
+        switch (ph) {  // uniform
+        case 1: return u32x4{a.w, b.x, b.y, b.z};
+        case 2: return u32x4{a.z, a.w, b.x, b.y};
+        default: return u32x4{a.y, a.z, a.w, b.x};
+        }
+    };
+    constexpr int kB = 4;
+    u32x4 cur = *reinterpret_cast<const u32x4*>(seg + 4 * (c_hi - 1));
+    for (int32_t c = c_hi - 1; c >= c_lo; c -= kB) {
+        u32x4 sv[kB];  // sources c-1 .. c-kB (all read before any of dests c .. c-kB+1 is written)
+#pragma unroll
+        for (int u = 0; u < kB; ++u) {
+            const int32_t i = c - 1 - u;
+            sv[u] = i >= c_lo ? *reinterpret_cast<const u32x4*>(seg + 4 * i) : below;
+        }
+#pragma unroll
+        for (int u = 0; u < kB; ++u) {
+            const int32_t d = c - u;
+            if (d >= c_lo) *reinterpret_cast<u32x4*>(seg + 4 * d) = comb(sv[u], u ? sv[u - 1] : cur);
+        }
+        cur = sv[kB - 1];
     }
 }
 
@@ -536,6 +602,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
     __shared__ uint32_t s_freed;         // output-ring words released by the storers (monotone)
     __shared__ uint32_t s_stages;        // free input stages (bit mask)
     __shared__ uint32_t s_alloc;         // ring positions whose ring decision is out
+    __shared__ uint32_t s_released;      // ring positions whose regions are released (storer groups)
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
@@ -551,6 +618,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
         s_freed = 0;
         s_stages = (1u << kStagesK) - 1u;
         s_alloc = 0;
+        s_released = 0;
         mbar_fence_init();
     }
     __syncthreads();
@@ -632,7 +700,10 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
         // chunked ballot ranker.
         const int g = warp / kGroupWarps, rw = warp % kGroupWarps;
         const int rt = tid - g * kRT;         // thread index within the group
-        const uint32_t gbar = 1 + 2 * g;      // named barrier of the group (2 is the storers')
+        // named barrier of the group (2 and 4 are the storers').  A register
+        // id here: one copy of the ranker loop per group (immediate ids) doubles
+        // the ranker code and measured -9 % at f = 0.5.
+        const uint32_t gbar = 1 + 2 * g;
         const int xs = kSeg * rw;
         const uint32_t smem_b = smem_addr(smem);
         const uint32_t ring_b = smem_addr(ring);
@@ -901,8 +972,15 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
         // aligned interior) plus <= 6 scalar head/tail words: the region is first
         // re-phased in shared memory so its words sit at their destination's
         // 16-byte phase.  The region is released once the bulk engine has read it.
-        const int st = tid - 32 * kWarpStorer0;
-        for (uint32_t k = 0;; ++k) {
+        constexpr int kSG = Layout<PART>::kStoreGroups;
+        const int sg = (tid - 32 * kWarpStorer0) / kST;  // storer group
+        const int st = (tid - 32 * kWarpStorer0) % kST;  // thread within the group
+        // one compiled copy of the loop per group, so the group's named barrier
+        // id is an immediate (a register id measured -12 % at f = 0.5)
+        auto storer_loop = [&](auto sg_tag) {
+        constexpr uint32_t kG = decltype(sg_tag)::value;
+        constexpr uint32_t sbar = kG ? 4u : 2u;         // the group's named barrier
+        for (uint32_t k = kG;; k += kSG) {
             const int o = k % kSlots;
             mbar_wait(&bar_resolved[o], (k / kSlots) & 1);
             const uint32_t t = meta[o].tile;
@@ -928,18 +1006,33 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             auto bulk_segment = [&](uint32_t* w0, uint32_t* base, uint64_t d0, uint32_t cnt) {
                 const uint64_t d1 = d0 + cnt;
                 const uint32_t sh = uint32_t(d0) & 3u;  // word r must sit at phase (d0 + r) & 3
-                if (sh) rephase<kST, Layout<PART>::kRephaseU>(w0, cnt, sh, st);
+                if (sh) {
+                    if (DS_IRR_REPHASE_RUNS) rephase_runs<kST>(w0, cnt, sh, st, sbar);
+                    else rephase<kST, Layout<PART>::kRephaseU>(w0, cnt, sh, st, sbar);
+                }
                 const uint32_t* const w = w0 + sh;
                 const uint64_t g0 = (d0 + 3) & ~3ull, g1 = d1 & ~3ull;
+#ifdef DS_TRACE_STORER
+                if (st == 0) trace_event(p.trace, t, 8, globaltimer());
+#endif
                 if (g1 > g0) {
                     fence_proxy_async_smem();  // re-phased words -> visible to the bulk engine
-                    named_bar_sync(2, kST);
+#ifdef DS_TRACE_STORER
+                    if (st == 0) trace_event(p.trace, t, 9, globaltimer());
+#endif
+                    named_bar_sync(sbar, kST);
+#ifdef DS_TRACE_STORER
+                    if (st == 0) trace_event(p.trace, t, 10, globaltimer());
+#endif
                     if (st == 0) bulk_s2g(base + g0, w + uint32_t(g0 - d0), uint32_t(g1 - g0) * 4u);
+#ifdef DS_TRACE_STORER
+                    if (st == 0) trace_event(p.trace, t, 11, globaltimer());
+#endif
                     if (st < 3 && d0 + st < g0) stg_stream(base + d0 + st, w[st]);
                     if (st >= 3 && st < 6 && g1 + (st - 3) < d1)
                         stg_stream(base + g1 + (st - 3), w[uint32_t(g1 - d0) + (st - 3)]);
                 } else {
-                    named_bar_sync(2, kST);
+                    named_bar_sync(sbar, kST);
                     if (uint32_t(st) < cnt) stg_stream(base + d0 + st, w[st]);  // cnt < 8
                 }
             };
@@ -955,18 +1048,35 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
                     if (F > 0) bulk_segment(seg + region_true(A), p.fbase, p.flo + ((vs0 - p.lo) - excl), F);
                 }
             }
-            named_bar_sync(2, kST);  // every storer is done with the region
+            // Every storer is done with the region.  With bulk stores only warp 0's
+            // lanes 0..7 (the scalar head / tail words) read it after the last
+            // barrier, so a warp sync orders them before lane 0's release.
+            if (kBulkStore && DS_IRR_STORE_WARP_SYNC) {
+                if (st < 32) __syncwarp();
+            } else {
+                named_bar_sync(sbar, kST);
+            }
             if (st == 0) {
                 trace_event(p.trace, t, 6, globaltimer());
                 bulk_commit();        // (possibly empty) group of this tile
                 bulk_wait_read<0>();  // the bulk engine has read the region
                 trace_event(p.trace, t, 12, globaltimer());
+                if (kSG > 1) {  // regions are released in ring order
+                    for (SpinGuard guard; ld_acquire_cta_smem(&s_released) != k;) {
+                        guard.check("irregular in-order release");
+                        __nanosleep(32);
+                    }
+                }
                 // ring words allocated up to this tile belong to tiles stored by now
                 st_release_cta_smem(&s_freed, ring_end);
                 if (!in_ring) stage_release(&s_stages, meta[o].stage);
                 mbar_arrive(&bar_stored[o]);
+                if (kSG > 1) st_release_cta_smem(&s_released, k + 1);
             }
         }
+        };
+        if (kSG > 1 && sg != 0) storer_loop(std::integral_constant<uint32_t, 1>{});
+        else storer_loop(std::integral_constant<uint32_t, 0>{});
         if (st == 0) bulk_wait_all();  // the bulk stores are complete before the CTA exits
     }
 }

@@ -54,6 +54,13 @@ def main():
     pct("resolved->storer", sstart - resolved)
     pct("rephase+issue", issued - sstart)
     pct("issue->released", released - issued)
+    if os.environ.get("DS_TRACE_STORER"):  # library built with -DDS_TRACE_STORER: sub-steps (slots 8-11)
+        sub = [us(c) for c in (8, 9, 10, 11)]
+        ok = (t[:, 8] > 0) & (t[:, 11] > 0)
+        for name, a, b in (("  start->rephased", sstart, sub[0]), ("  rephased->fenced", sub[0], sub[1]),
+                           ("  fenced->barrier", sub[1], sub[2]), ("  barrier->issued", sub[2], sub[3]),
+                           ("  bulk issued->end", sub[3], issued)):
+            pct(name, (b - a)[ok])
     pct("draw->released", released - drawn)
     sm = t[:, 7] & 0xffff
     busy, life = [], []
