@@ -121,9 +121,14 @@ __device__ __forceinline__ void stg_stream(uint32_t* p, uint32_t a) {
 // {ticket, epoch}.  A launch makes exactly `draws` draws in total (the
 // persistent kernels: ntiles + gridDim.x, every CTA's last draw fails); the
 // CTA that makes the final draw re-arms the word for the next launch.
-__device__ __forceinline__ void draw_ticket(uint64_t* ctrl, uint32_t draws, uint32_t& ticket,
-                                            uint32_t& epoch) {
-    unsigned long long old = atomicAdd(reinterpret_cast<unsigned long long*>(ctrl), 1ull);
+// Split form: issue_ticket() sends the atomic (the caller can overlap its
+// round trip with other work, e.g. the barrier set-up at kernel entry);
+// take_ticket() decodes it and re-arms the word after the launch's last draw.
+__device__ __forceinline__ unsigned long long issue_ticket(uint64_t* ctrl) {
+    return atomicAdd(reinterpret_cast<unsigned long long*>(ctrl), 1ull);
+}
+__device__ __forceinline__ void take_ticket(uint64_t* ctrl, uint32_t draws, unsigned long long old,
+                                            uint32_t& ticket, uint32_t& epoch) {
     ticket = uint32_t(old);
     epoch = uint32_t(old >> 32);
     if (ticket == draws - 1) {
@@ -131,6 +136,10 @@ __device__ __forceinline__ void draw_ticket(uint64_t* ctrl, uint32_t draws, uint
         if ((ne & kEpochMask) == 0) ne++;  // epoch 0 is never valid (zeroed status)
         atomicExch(reinterpret_cast<unsigned long long*>(ctrl), (unsigned long long)ne << 32);
     }
+}
+__device__ __forceinline__ void draw_ticket(uint64_t* ctrl, uint32_t draws, uint32_t& ticket,
+                                            uint32_t& epoch) {
+    take_ticket(ctrl, draws, issue_ticket(ctrl), ticket, epoch);
 }
 
 // ---- shared-memory mbarrier + 1-D TMA bulk copy (cp.async.bulk) --------
@@ -255,6 +264,12 @@ __device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity, ui
 // Named barrier among `count` threads (a subset of the CTA, whole warps).
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t count) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+// Arrive on a named barrier without waiting (producer side of a bar.arrive /
+// bar.sync pair: the arriving thread's prior writes are ordered before the
+// waiters' later accesses).
+__device__ __forceinline__ void named_bar_arrive(uint32_t id, uint32_t count) {
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(count) : "memory");
 }
 
 // Global -> shared bulk copy of `bytes` (multiple of 16, both addresses

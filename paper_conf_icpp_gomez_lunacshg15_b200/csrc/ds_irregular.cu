@@ -63,6 +63,7 @@ struct IrregParams {
     uint32_t value_hi;  // 8-byte elements: high word of the value / parameter
     uint32_t wshift;    // out_n = words >> wshift (1 for 8-byte elements)
     uint64_t* trace;  // diagnostics: per-tile events, or null
+    uint64_t* trace_cta;  // diagnostics: per-CTA events (after the tiles' events), or null
     uint32_t* tbase;  // 16-byte-aligned base of the true/kept output (== abase in place)
     uint64_t tlo;     // its word offset (output word j lives at tbase[tlo + j])
     uint32_t* fbase;  // same for the false words (partition), or null
@@ -678,8 +679,21 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
     __shared__ uint32_t s_released;      // ring positions whose regions are released (storer groups)
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // per-CTA diagnostics: 0 entry, 1 initialised, 2 producer done, 3/4 storer
+    // groups done, 5/6 ranker groups done, 7.. resolvers done; 15 SM id
+    auto trace_cta = [&](int ev) { trace_event(p.trace_cta, blockIdx.x, ev, globaltimer()); };
     if (tid == 0) {
-        for (int o = 0; o < kSlots; ++o) {
+        trace_cta(0);
+        trace_event(p.trace_cta, blockIdx.x, 15, smid());
+    }
+    // The producer warp sets up the barriers (one slot per lane) while its lane
+    // 0's first ticket atomic (one L2 round trip) is in flight, then ARRIVES on
+    // the start barrier and goes on to its first load; the other warps wait on
+    // it (bar.arrive / bar.sync: the set-up is ordered before their accesses).
+    unsigned long long first_old = 0;
+    if (warp == kWarpProducer) {
+        if (lane == 0) first_old = issue_ticket(p.ctrl);
+        for (int o = lane; o < kSlots; o += 32) {
             mbar_init(&bar_loaded[o], 1);
             mbar_init(&bar_drawn[o], 1);
             mbar_init(&bar_counted[o], 1);
@@ -687,14 +701,20 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             mbar_init(&bar_resolved[o], 1);
             mbar_init(&bar_stored[o], 1);
         }
-        s_end = 0xffffffffu;
-        s_freed = 0;
-        s_stages = (1u << kStagesK) - 1u;
-        s_alloc = 0;
-        s_released = 0;
-        mbar_fence_init();
+        if (lane == 0) {
+            s_end = 0xffffffffu;
+            s_freed = 0;
+            s_stages = (1u << kStagesK) - 1u;
+            s_alloc = 0;
+            s_released = 0;
+        }
+        if (lane < kSlots) mbar_fence_init();
+        __syncwarp();
+        named_bar_arrive(0, Layout<PART>::kThreads);
+    } else {
+        named_bar_sync(0, Layout<PART>::kThreads);
     }
-    __syncthreads();
+    if (tid == 0) trace_cta(1);
 
     if (warp == kWarpProducer) {
         // ------------------------------------------------ producer (lane 0)
@@ -715,21 +735,29 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             atomicAnd(&s_stages, ~(1u << s));
             uint32_t* stage = smem + s * kStageWords;
             uint32_t t, epoch;
-            draw_ticket(p.ctrl, p.draws, t, epoch);
-            if (k == 0) s_epoch = epoch;
+            if (k > 0) {
+                draw_ticket(p.ctrl, p.draws, t, epoch);
+            } else {
+                take_ticket(p.ctrl, p.draws, first_old, t, epoch);
+                s_epoch = epoch;
+            }
             if (t >= p.ntiles) {  // one failed draw per CTA ends its work
                 meta[o].tile = kNoTile;
                 st_release_cta_smem(&s_end, k);
                 mbar_arrive(&bar_drawn[o]);
                 mbar_arrive(&bar_loaded[o]);
-                // End markers for the other resolvers' next positions, so each of
-                // them finds one and no warp has to poll for the end of the work.
+                // End markers for the other resolvers' (and ranker groups') next
+                // positions, so each of them finds one and no warp has to poll
+                // for the end of the work.
+                static_assert(kRankGroups <= kResolvers, "end markers");
                 for (uint32_t j = 1; j < uint32_t(kResolvers); ++j) {
                     const uint32_t kj = k + j, oj = kj % kSlots;
                     mbar_wait(&bar_stored[oj], ((kj / kSlots) & 1) ^ 1);
                     meta[oj].tile = kNoTile;
                     mbar_arrive(&bar_drawn[oj]);
+                    if (j < uint32_t(kRankGroups)) mbar_arrive(&bar_loaded[oj]);
                 }
+                trace_cta(2);
                 return;
             }
             meta[o].tile = t;
@@ -785,9 +813,15 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
         if (Op::kUnique && !Op::kWide) has_hprev = halo_prev(p, hprev);
         for (uint32_t k = g;; k += kRankGroups) {
             const int o = k % kSlots;
-            if (!mbar_wait_or_end(&bar_loaded[o], (k / kSlots) & 1, &s_end, k)) break;
+            if (!mbar_wait_or_end(&bar_loaded[o], (k / kSlots) & 1, &s_end, k)) {
+                if (rt == 0) trace_cta(5 + g);
+                break;
+            }
             const uint32_t t = meta[o].tile;
-            if (t == kNoTile) break;
+            if (t == kNoTile) {
+                if (rt == 0) trace_cta(5 + g);
+                break;
+            }
             const uint32_t s = meta[o].stage;
             if (rt == 0) trace_event(p.trace, t, 1, globaltimer());
             const uint64_t tb = uint64_t(t) * kT;
@@ -1009,7 +1043,10 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             mbar_wait(&bar_drawn[o], use & 1);  // a tile, or an end marker (every resolver gets one)
             const uint32_t t = meta[o].tile;
             if (t == kNoTile) {
-                if (lane == 0) mbar_arrive(&bar_resolved[o]);
+                if (lane == 0) {
+                    mbar_arrive(&bar_resolved[o]);
+                    trace_cta(7 + r);
+                }
                 break;
             }
             const uint32_t epoch = s_epoch;
@@ -1152,7 +1189,10 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
         };
         if (kSG > 1 && sg != 0) storer_loop(std::integral_constant<uint32_t, 1>{});
         else storer_loop(std::integral_constant<uint32_t, 0>{});
-        if (st == 0) bulk_wait_all();  // the bulk stores are complete before the CTA exits
+        if (st == 0) {
+            bulk_wait_all();  // the bulk stores are complete before the CTA exits
+            trace_cta(3 + sg);
+        }
     }
 }
 
@@ -1182,6 +1222,7 @@ cudaError_t launch_op(IrregParams p, cudaStream_t s) {
     uint64_t grid = uint64_t(lc.sms) * lc.per_sm;
     if (grid > p.ntiles) grid = p.ntiles;
     p.draws = p.ntiles + uint32_t(grid);
+    if (p.trace && debug_trace(size_t(p.ntiles) + grid)) p.trace_cta = p.trace + size_t(p.ntiles) * kTraceWords;
     kern<<<uint32_t(grid), Layout<PART>::kThreads, kSmem, s>>>(p);
     return cudaGetLastError();
 }

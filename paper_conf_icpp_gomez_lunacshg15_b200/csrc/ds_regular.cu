@@ -221,6 +221,9 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
     __shared__ StageMeta meta[kStages];
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // The first ticket's atomic is in flight while thread 0 sets up the barriers.
+    unsigned long long first_old = 0;
+    if (tid == 0) first_old = issue_ticket(p.ctrl);
     if (tid == 0) {
         for (int s = 0; s < kStages; ++s) {
             mbar_init(&bar_full[s], 32);  // every producer lane arrives (its stage writes, slow path)
@@ -242,7 +245,10 @@ __global__ void __launch_bounds__(kThreads, 2) regular_kernel(const RegParams p)
             uint32_t* stage = smem + s * kStageWords;
             mbar_wait(&bar_empty[s], (use & 1) ^ 1);  // consumers released tile k - kStages
             uint32_t t = 0, epoch = 0;
-            if (lane == 0) draw_ticket(p.ctrl, p.draws, t, epoch);
+            if (lane == 0) {
+                if (k == 0) take_ticket(p.ctrl, p.draws, first_old, t, epoch);
+                else draw_ticket(p.ctrl, p.draws, t, epoch);
+            }
             t = __shfl_sync(0xffffffffu, t, 0);
             epoch = __shfl_sync(0xffffffffu, epoch, 0);
             if (t >= p.ntiles) {  // one failed draw per CTA ends its work

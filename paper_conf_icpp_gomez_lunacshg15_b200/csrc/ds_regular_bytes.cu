@@ -218,6 +218,9 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
     __shared__ uint32_t geo_epoch[kBStages];
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    // The first ticket's atomic is in flight while thread 0 sets up the barriers.
+    unsigned long long first_old = 0;
+    if (tid == 0) first_old = issue_ticket(p.ctrl);
     if (tid == 0) {
         for (int s = 0; s < kBStages; ++s) {
             mbar_init(&bar_full[s], 32);  // every producer lane arrives (its stage writes, slow path)
@@ -236,7 +239,10 @@ __global__ void __launch_bounds__(kBThreads, 2) regular_bytes_kernel(const RegBP
             uint8_t* stage = smem8 + size_t(s) * kBStageAlloc;
             mbar_wait(&bar_empty[s], ((k / kBStages) & 1) ^ 1);
             uint32_t t = 0, epoch = 0;
-            if (lane == 0) draw_ticket(p.ctrl, p.draws, t, epoch);
+            if (lane == 0) {
+                if (k == 0) take_ticket(p.ctrl, p.draws, first_old, t, epoch);
+                else draw_ticket(p.ctrl, p.draws, t, epoch);
+            }
             t = __shfl_sync(0xffffffffu, t, 0);
             epoch = __shfl_sync(0xffffffffu, epoch, 0);
             if (t >= p.ntiles) {
