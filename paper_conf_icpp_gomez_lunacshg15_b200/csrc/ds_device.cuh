@@ -286,6 +286,12 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
         : "memory");
 }
 
+// L2 prefetch of `bytes` (multiple of 16, 16-byte aligned) global bytes: the
+// bulk engine reads them into L2 without a destination or completion.
+__device__ __forceinline__ void bulk_prefetch_l2(const void* src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+
 // Shared -> global bulk copy (TMA store) of `bytes` (multiple of 16, both
 // addresses 16-byte aligned), tracked by the issuing thread's bulk async-group.
 __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {

@@ -340,6 +340,16 @@ constexpr uint32_t kDropTile = DS_DEBUG_DROP_TILE;
 #define DS_IRR_LATE_LB 0
 #endif
 constexpr int kLateLookback = DS_IRR_LATE_LB;  // look-back starts at: 0 the draw, 1 the own AGG, 2 the tile's landing
+// L2 prefetch of the tile DS_IRR_PREFETCH grids ahead of each drawn ticket (0:
+// off), while the CTA's last counted tile kept >= DS_IRR_PREFETCH_MIN_KEEP words
+// (producer loop)
+#ifndef DS_IRR_PREFETCH
+#define DS_IRR_PREFETCH 1
+#endif
+constexpr uint32_t kPrefetchDist = DS_IRR_PREFETCH;
+#ifndef DS_IRR_PREFETCH_MIN_KEEP
+#define DS_IRR_PREFETCH_MIN_KEEP 3686  // 45 % of a tile
+#endif
 
 __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint32_t tile,
                                              uint32_t epoch, int lane, uint64_t* trace) {
@@ -677,6 +687,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
     __shared__ uint32_t s_stages;        // free input stages (bit mask)
     __shared__ uint32_t s_alloc;         // ring positions whose ring decision is out
     __shared__ uint32_t s_released;      // ring positions whose regions are released (storer groups)
+    __shared__ uint32_t s_recent_total;  // kept words of the CTA's most recently counted tile (prefetch policy)
 
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     // per-CTA diagnostics: 0 entry, 1 initialised, 2 producer done, 3/4 storer
@@ -707,6 +718,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             s_stages = (1u << kStagesK) - 1u;
             s_alloc = 0;
             s_released = 0;
+            s_recent_total = 0;
         }
         if (lane < kSlots) mbar_fence_init();
         __syncwarp();
@@ -719,29 +731,37 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
     if (warp == kWarpProducer) {
         // ------------------------------------------------ producer (lane 0)
         if (lane != 0) return;
-        for (uint32_t k = 0;; ++k) {
-            const int o = k % kSlots;
-            mbar_wait(&bar_stored[o], ((k / kSlots) & 1) ^ 1);  // slot o finished tile k - kSlots
-            // any free input stage (a tile compacted into the ring frees its stage at
-            // once, one compacted in place only once stored)
+        // Free input stages: a tile compacted into the ring frees its stage at
+        // once, one compacted in place only once stored.
+        auto claim_stage = [&]() -> uint32_t {
             uint32_t m;
             SpinGuard guard;
-            const uint64_t t_claim = p.trace ? globaltimer() : 0;  // diagnostics: stage wait
             while ((m = ld_acquire_cta_smem(&s_stages)) == 0u) {
                 guard.check("irregular producer stage wait");
                 __nanosleep(32);
             }
             const uint32_t s = __ffs(m) - 1;
             atomicAnd(&s_stages, ~(1u << s));
+            return s;
+        };
+        // Position k's ticket is drawn only once slot k and a stage are free, so a
+        // drawn tile never waits for anything but its own load (a drawn tile that
+        // waited would hold up every later tile's look-back: a convoy; drawing
+        // the next ticket as soon as a second stage is free measured -3 to -7 %,
+        // DESIGN.md §7).
+        uint64_t claim_cur = p.trace ? globaltimer() : 0;  // diagnostics: stage wait start
+        uint32_t s_cur = claim_stage();
+        unsigned long long old_cur = first_old;  // issued at kernel entry
+        bool pf_on = DS_IRR_PREFETCH_MIN_KEEP == 0;  // L2 prefetch policy (see the end of the loop)
+        for (uint32_t k = 0;; ++k) {
+            const int o = k % kSlots;
+            const uint32_t s = s_cur;
+            const uint64_t t_claim = claim_cur;
             uint32_t* stage = smem + s * kStageWords;
             uint32_t t, epoch;
-            if (k > 0) {
-                draw_ticket(p.ctrl, p.draws, t, epoch);
-            } else {
-                take_ticket(p.ctrl, p.draws, first_old, t, epoch);
-                s_epoch = epoch;
-            }
-            if (t >= p.ntiles) {  // one failed draw per CTA ends its work
+            take_ticket(p.ctrl, p.draws, old_cur, t, epoch);
+            if (k == 0) s_epoch = epoch;
+            if (t >= p.ntiles) {  // a failed draw ends the CTA's work
                 meta[o].tile = kNoTile;
                 st_release_cta_smem(&s_end, k);
                 mbar_arrive(&bar_drawn[o]);
@@ -785,6 +805,34 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             fence_proxy_async_smem();
             mbar_arrive_expect_tx(&bar_loaded[o], bytes);
             if (bytes) bulk_g2s(dst, p.abase + beg, bytes, &bar_loaded[o]);
+            if (kPrefetchDist && !PART && pf_on) {
+                // L2 prefetch of the tile kPrefetchDist grids ahead: tickets are drawn
+                // in order by all CTAs, so that tile is drawn ~1-3 us from now and its
+                // load then hits L2 (each tile is prefetched once, by the CTA that drew
+                // the ticket kPrefetchDist * grid before it).  No lower tile ever
+                // writes into a higher tile's input (§4.3), so the lines stay current.
+                const uint64_t tp = uint64_t(t) + uint64_t(kPrefetchDist) * gridDim.x;
+                if (tp < p.ntiles) {
+                    const uint64_t pb = tp * kT - ((Op::kUnique && tp > 0) ? kPre : 0);
+                    const uint64_t pe = (tp * kT + kT < p.hi ? tp * kT + kT : p.hi) & ~3ull;
+                    if (pe > pb) bulk_prefetch_l2(p.abase + pb, uint32_t(pe - pb) * 4u);
+                }
+            }
+            // the next position's ticket: once its slot and a stage are free
+            {
+                const uint32_t k1 = k + 1, o1 = k1 % kSlots;
+                mbar_wait(&bar_stored[o1], ((k1 / kSlots) & 1) ^ 1);  // slot o1 finished tile k1 - kSlots
+                claim_cur = p.trace ? globaltimer() : 0;
+                s_cur = claim_stage();
+                old_cur = issue_ticket(p.ctrl);
+            }
+            // The prefetch policy for the next tile, decided off the critical path
+            // (the next ticket's round trip is in flight): prefetch only while the
+            // CTA's last counted tile kept >= DS_IRR_PREFETCH_MIN_KEEP words.  At
+            // low keep fractions the producer loop, not the input stages, bounds
+            // the rate, and the prefetch does not pay.
+            if (kPrefetchDist && DS_IRR_PREFETCH_MIN_KEEP)
+                pf_on = *static_cast<volatile uint32_t*>(&s_recent_total) >= uint32_t(DS_IRR_PREFETCH_MIN_KEEP);
         }
     } else if (warp < kRankWarps) {
         // ------------------------------------------------ ranker warps
@@ -947,6 +995,8 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
                 // a4: publish the aggregate right away -- it depends on nothing else
                 // (a relaxed status store).
                 meta[o].total = total;
+                if (kPrefetchDist && DS_IRR_PREFETCH_MIN_KEEP)
+                    *static_cast<volatile uint32_t*>(&s_recent_total) = total;  // a hint only
                 debug_delay(t, 1);
                 if (t != kDropTile)
                     publish_status(status_ptr(p.status, t), make_status(t == 0 ? kStateIncl : kStateAgg, s_epoch, total));

@@ -38,10 +38,21 @@ def main():
     hold = (t[:, 15] - t[:, 0]) / 1e3
     land = (t[:, 1] - t[:, 0]) / 1e3
     span = (t[:, 6].max() - t[:, 0].min()) / 1e3
-    print(f"n=2^{lg} f={f} tiles={ntiles} rate={ntiles / span:.1f} tiles/us; in ring {in_ring.mean():.1%}")
-    for name, d in (("stage wait", wait), ("draw->landed", land), ("draw->ranked", hold)):
+    print(f"n=2^{lg} f={f} tiles={ntiles} rate={ntiles / span:.1f} tiles/us; in ring {in_ring.mean():.1%}"
+          " ('stage wait' = claim -> drawn: the wait for a free stage + the ticket atomic)")
+    # producer loop, per CTA in draw order: after a draw until the next claim
+    # starts (load issue, slot wait) and claim -> draw (stage wait + ticket atomic)
+    sm = t[:, 7] & 0xffff
+    post = []
+    for s_ in np.unique(sm):
+        idx = np.where(sm == s_)[0]
+        idx = idx[np.argsort(t[idx, 0])]
+        post.append((t[idx[1:], 13] - t[idx[:-1], 0]) / 1e3)
+    post = np.concatenate(post)
+    for name, d in (("stage wait", wait), ("draw->landed", land), ("draw->ranked", hold),
+                    ("draw->next claim", post)):
         q = np.percentile(d, [5, 50, 95])
-        print(f"{name:13s} p5 {q[0]:6.2f} p50 {q[1]:6.2f} p95 {q[2]:6.2f} mean {d.mean():6.2f} us")
+        print(f"{name:16s} p5 {q[0]:6.2f} p50 {q[1]:6.2f} p95 {q[2]:6.2f} mean {d.mean():6.2f} us")
 
 
 if __name__ == "__main__":
