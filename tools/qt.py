@@ -113,6 +113,17 @@ def run(spec):
         aux = torch.empty_like(a)
         timeit(f"partition 256M f={f}", a, lambda w, d: libds.ds_partition_ex(w, n, 1, t, aux, d, None),
                lambda m: 4 * (2 * n + 2 * (n - m)))
+    elif op in ("padbig", "unpadbig", "padbig8"):  # >= 256M elements, word kernel
+        R, C, NC = 16384, 16383, 16384
+        eb = 8 if op == "padbig8" else 4
+        a = dsgen.matrix_input(R, C, NC, eb, device=dev)
+        if op.startswith("pad"):
+            timeit(f"pad {R}x{C}->{NC} eb={eb}", a, lambda w, d: libds.ds_pad_ex(w, R, C, NC, eb, None, None),
+                   lambda m: eb * (R * C + R * NC))
+        else:
+            libds.ds_pad(a, R, C, NC, eb)
+            timeit(f"unpad {R}x{NC}->{C} eb={eb}", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, eb, None),
+                   lambda m: eb * (2 * R * C))
     elif op == "pad12k":
         R, C, NC = 12000, 11999, 12000
         a = dsgen.matrix_input(R, C, NC, 4, device=dev)
