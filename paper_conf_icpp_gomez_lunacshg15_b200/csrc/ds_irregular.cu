@@ -250,6 +250,8 @@ struct SmemSplit {
     static_assert(kSlots >= kStages && kStages <= 32, "stages");
 };
 static_assert(kSlots % kResolvers == 0, "a slot is always served by the same resolver");
+static_assert(kSlots % kRankGroups == 0 && kSlots % 2 == 0,
+              "a slot is always served by the same ranker group and storer group");
 static_assert(kSmem + kStaticSmem <= 227 * 1024, "shared memory");
 
 struct SlotMeta {
