@@ -349,6 +349,9 @@ constexpr int kLateLookback = DS_IRR_LATE_LB;  // look-back starts at: 0 the dra
 #define DS_IRR_PREFETCH 1
 #endif
 constexpr uint32_t kPrefetchDist = DS_IRR_PREFETCH;
+#ifndef DS_IRR_PART_PREFETCH
+#define DS_IRR_PART_PREFETCH 0  // partition stores every word of a tile: no keep-fraction policy
+#endif
 #ifndef DS_IRR_PREFETCH_MIN_KEEP
 #define DS_IRR_PREFETCH_MIN_KEEP 3686  // 45 % of a tile
 #endif
@@ -574,10 +577,16 @@ __device__ __forceinline__ void rephase(uint32_t* seg, uint32_t cnt, uint32_t ph
 #ifndef DS_IRR_STORE_WARP_SYNC
 #define DS_IRR_STORE_WARP_SYNC 1
 #endif
+#ifndef DS_IRR_REPHASE_BATCH
+#define DS_IRR_REPHASE_BATCH 4  // chunks read ahead per thread in rephase_runs (compaction, select, unique)
+#endif
+#ifndef DS_IRR_PART_REPHASE_BATCH
+#define DS_IRR_PART_REPHASE_BATCH 2  // the same for partition (72 registers; measured 2 > 4 > 8)
+#endif
 #ifndef DS_IRR_REPHASE_RUNS
 #define DS_IRR_REPHASE_RUNS 1
 #endif
-template <int kSTT>
+template <int kSTT, int kB>
 __device__ __forceinline__ void rephase_runs(uint32_t* seg, uint32_t cnt, uint32_t ph, int st,
                                              uint32_t bar) {
     const int32_t nchunks = int32_t((cnt + ph + 3) >> 2);
@@ -597,7 +606,6 @@ __device__ __forceinline__ void rephase_runs(uint32_t* seg, uint32_t cnt, uint32
         default: return u32x4{a.y, a.z, a.w, b.x};
         }
     };
-    constexpr int kB = 4;
     u32x4 cur = *reinterpret_cast<const u32x4*>(seg + 4 * (c_hi - 1));
     for (int32_t c = c_hi - 1; c >= c_lo; c -= kB) {
         u32x4 sv[kB];  // sources c-1 .. c-kB (all read before any of dests c .. c-kB+1 is written)
@@ -807,7 +815,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             fence_proxy_async_smem();
             mbar_arrive_expect_tx(&bar_loaded[o], bytes);
             if (bytes) bulk_g2s(dst, p.abase + beg, bytes, &bar_loaded[o]);
-            if (kPrefetchDist && !PART && pf_on) {
+            if (kPrefetchDist && (PART ? DS_IRR_PART_PREFETCH : pf_on)) {
                 // L2 prefetch of the tile kPrefetchDist grids ahead: tickets are drawn
                 // in order by all CTAs, so that tile is drawn ~1-3 us from now and its
                 // load then hits L2 (each tile is prefetched once, by the CTA that drew
@@ -1171,7 +1179,7 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
                 const uint64_t d1 = d0 + cnt;
                 const uint32_t sh = uint32_t(d0) & 3u;  // word r must sit at phase (d0 + r) & 3
                 if (sh) {
-                    if (DS_IRR_REPHASE_RUNS) rephase_runs<kST>(w0, cnt, sh, st, sbar);
+                    if (DS_IRR_REPHASE_RUNS) rephase_runs<kST, PART ? DS_IRR_PART_REPHASE_BATCH : DS_IRR_REPHASE_BATCH>(w0, cnt, sh, st, sbar);
                     else rephase<kST, Layout<PART>::kRephaseU>(w0, cnt, sh, st, sbar);
                 }
                 const uint32_t* const w = w0 + sh;

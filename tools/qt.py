@@ -124,6 +124,13 @@ def run(spec):
             libds.ds_pad(a, R, C, NC, eb)
             timeit(f"unpad {R}x{NC}->{C} eb={eb}", a, lambda w, d: libds.ds_unpad_ex(w, R, NC, C, eb, None),
                    lambda m: eb * (2 * R * C))
+    elif op == "partcopy":  # the partition's DS pass alone, out of place (trues and falses)
+        n = 1 << 28
+        a = dsgen.select_input(n, dsgen.seed_for(5), device=dev)
+        t = dsgen.select_threshold(f) & 0xFFFFFFFF
+        ot, of = torch.empty_like(a), torch.empty_like(a)
+        timeit(f"partition_copy 256M f={f}", a,
+               lambda w, d: libds.ds_partition_copy_ex(w, n, 1, t, ot, of, d, None), lambda m: 4 * (2 * n))
     elif op == "pad12k":
         R, C, NC = 12000, 11999, 12000
         a = dsgen.matrix_input(R, C, NC, 4, device=dev)

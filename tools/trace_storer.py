@@ -27,8 +27,14 @@ def main():
     n = 1 << lg
     T = libds.ds_tile_size(libds.DS_KERNEL_IRREGULAR)
     op = os.environ.get("DS_OP", "compact")
-    src = dsgen.unique_runs_input(n, f, 5, device="cuda") if op == "unique" else \
-        dsgen.compact_input(n, f, 7, device="cuda")
+    if op == "unique":
+        src = dsgen.unique_runs_input(n, f, 5, device="cuda")
+    elif op == "partcopy":  # the partition's DS pass, out of place
+        src = dsgen.select_input(n, dsgen.seed_for(5), device="cuda")
+        thr = dsgen.select_threshold(f) & 0xFFFFFFFF
+        ot, of = torch.empty_like(src), torch.empty_like(src)
+    else:
+        src = dsgen.compact_input(n, f, 7, device="cuda")
     work = torch.empty_like(src)
     ntiles = (n + T - 1) // T
     tr = torch.zeros(ntiles * 16, dtype=torch.int64, device="cuda")
@@ -39,6 +45,8 @@ def main():
         libds.ds_debug_set_trace(tr if rep == 2 else None, ntiles if rep == 2 else 0)
         if op == "unique":
             libds.ds_unique_ex(work, n, None, 0, d_n, None)
+        elif op == "partcopy":
+            libds.ds_partition_copy_ex(work, n, 1, thr, ot, of, d_n, None)
         else:
             libds.ds_compact_ex(work, n, 0, d_n, None)
         torch.cuda.synchronize()
