@@ -49,6 +49,12 @@ def main():
         idx = idx[np.argsort(t[idx, 0])]
         post.append((t[idx[1:], 13] - t[idx[:-1], 0]) / 1e3)
     post = np.concatenate(post)
+    if os.environ.get("DS_TRACE_PRODUCER"):  # library built with -DDS_TRACE_PRODUCER: slots 8-11
+        for name, a, b in (("claim->taken", 13, 8), ("taken->drawn", 8, 0), ("drawn->pre-fence", 0, 9),
+                           ("fence", 9, 10), ("bulk issue", 10, 11)):
+            d = (t[:, b] - t[:, a]) / 1e3
+            q = np.percentile(d, [5, 50, 95])
+            print(f"  {name:16s} p5 {q[0]:6.2f} p50 {q[1]:6.2f} p95 {q[2]:6.2f} mean {d.mean():6.2f} us")
     for name, d in (("stage wait", wait), ("draw->landed", land), ("draw->ranked", hold),
                     ("draw->next claim", post)):
         q = np.percentile(d, [5, 50, 95])
