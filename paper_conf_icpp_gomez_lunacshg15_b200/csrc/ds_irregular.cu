@@ -367,7 +367,11 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
         int64_t idx = base - lane;
         uint64_t s = idx >= 0 ? ld_relaxed_gpu(status_ptr(status, idx)) : make_status(kStateIncl, epoch, 0);
         bool ok = status_current(s, epoch);
+#ifndef DS_TRACE_PRODUCER
         if (rounds++ == 0 && lane == 0) trace_event(trace, tile, 10, globaltimer());
+#else
+        ++rounds;
+#endif
         uint32_t L;  // nearest INCL at lane L (32: none this round)
         while (true) {
             const uint32_t inclm = __ballot_sync(kFull, ok && status_state(s) == kStateIncl);
@@ -391,11 +395,13 @@ __device__ __forceinline__ uint64_t lookback(uint64_t* __restrict__ status, uint
         }
         base -= 32;
     }
+#ifndef DS_TRACE_PRODUCER
     if (lane == 0) {
         trace_event(trace, tile, 8, rounds);
         trace_event(trace, tile, 9, polls);
         trace_event(trace, tile, 11, globaltimer());
     }
+#endif
     lookback_acquire();
     __syncwarp();
     return excl;
@@ -697,6 +703,9 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             uint32_t* stage = smem + s * kStageWords;
             uint32_t t, epoch;
             take_ticket(p.ctrl, p.draws, old_cur, t, epoch);
+#ifdef DS_TRACE_PRODUCER
+            const uint64_t tp_taken = globaltimer();
+#endif
             if (k == 0) s_epoch = epoch;
             if (t >= p.ntiles) {  // a failed draw ends the CTA's work
                 meta[o].tile = kNoTile;
@@ -739,9 +748,19 @@ __global__ void __launch_bounds__(Layout<PART>::kThreads, 1) irregular_kernel(co
             for (uint64_t w = end16 > beg ? end16 : beg; w < end; ++w)
                 dst[w - beg] = ldg_stream(p.abase + w);  // before the arrival that publishes the stage
             const uint32_t bytes = end16 > beg ? uint32_t(end16 - beg) * 4u : 0u;
+#ifdef DS_TRACE_PRODUCER  // producer sub-steps in slots 8-11 (the look-back's diagnostics are off)
+            trace_event(p.trace, t, 8, tp_taken);
+            trace_event(p.trace, t, 9, globaltimer());
+#endif
             fence_proxy_async_smem();
+#ifdef DS_TRACE_PRODUCER
+            trace_event(p.trace, t, 10, globaltimer());
+#endif
             mbar_arrive_expect_tx(&bar_loaded[o], bytes);
             if (bytes) bulk_g2s(dst, p.abase + beg, bytes, &bar_loaded[o]);
+#ifdef DS_TRACE_PRODUCER
+            trace_event(p.trace, t, 11, globaltimer());
+#endif
             if (kPrefetchDist && (PART ? DS_IRR_PART_PREFETCH : pf_on)) {
                 // L2 prefetch of the tile kPrefetchDist grids ahead: tickets are drawn
                 // in order by all CTAs, so that tile is drawn ~1-3 us from now and its
