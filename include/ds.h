@@ -302,7 +302,11 @@ uint64_t ds_launch_count(void);
  * bulk engine has read the stored region (irregular; region released);
  * 13 the producer starts waiting for a free input stage, 14 after the
  * ranker barrier, 15 compacted; 7 also carries bit 16 = compacted into the
- * output ring (else in place)).
+ * output ring (else in place)).  When capacity_tiles also covers the grid
+ * (ntiles + number of CTAs), the irregular kernels record per-CTA events in
+ * the words after the tiles' (CTA b at tile index ntiles + b: 0 entry,
+ * 1 set up, 2 producer done, 3/4 storer groups done, 5/6 ranker groups done,
+ * 7.. resolvers done, 15 SM id; tools/trace_cta.py).
  * NULL disables.  Development aid for DESIGN.md §7, not used by the API.  */
 ds_status ds_debug_set_trace(uint64_t* d_trace, size_t capacity_tiles);
 /* Library version, major*10000 + minor*100 + patch.                      */
